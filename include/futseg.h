@@ -1,0 +1,227 @@
+/*
+ * futseg.h -- C ABI of libfutseg, the B200 (sm_100a) hot path of Futhark's
+ * compiled code (Henriksen et al., PLDI'17; /root/reference/PAPER.md = "L<n>").
+ *
+ * After fusion (Sec. 4) and flattening (Sec. 5) a Futhark program is a perfect
+ * map nest whose innermost operator is a reduce, a scan or a stream_red.
+ * This library implements those innermost operators as hand-written CUDA
+ * kernels, over a fixed operator table:
+ *
+ *   op     : FS_ADD, FS_MIN, FS_MAX, FS_ARGMIN (value + index), FS_VADD (k-wide
+ *            vector add, the map(+) operator of Fig 4b/4c and G5)
+ *   dtype  : FS_I32, FS_I64, FS_F32
+ *   map f  : FS_MAP_ID, FS_MAP_NN_DIST (Rodinia NN distance, see fs_mapdesc)
+ *
+ * Semantics (each a plain definition; the oracle in oracle/ is that definition):
+ *   reduce (+) 0(+) [a1..an] = 0(+) (+) a1 (+) ... (+) an            L127-128
+ *   scan   (+) 0(+) [a1..an] = [a1, ..., a1 (+) ... (+) an] (inclusive) L129-130
+ *   redomap  = fold (+,0(+)) f = reduce (+) . map f                   L240-241, L254
+ *   scanomap = scan (+) . map f   (name by analogy with redomap, L978)
+ *   stream_red (map(+)) over chunks, each chunk folding into a fresh
+ *   zero accumulator in place                       Fig 4c, Fig 8
+ *   seg_reduce / seg_scan = map (reduce/scan) over the rows of a regular
+ *   [nseg][seglen] array ("segmented" scan/reduce)  footnote 5 L1230-1233
+ *   transpose_2d = rearrange (1,0) / as_column_major             L1389-1393, L1431
+ *
+ * Operator readings:
+ *   - integer ADD wraps modulo 2^32 / 2^64 (two's complement);
+ *   - neutral elements: ADD 0, MIN +inf / INT_MAX, MAX -inf / INT_MIN,
+ *     ARGMIN (MIN's neutral, index -1);
+ *   - ARGMIN is the lexicographic minimum of (value, index): among equal
+ *     values the smallest index wins (first occurrence);
+ *   - all operators are associative and commutative, so kernels may
+ *     reassociate and reorder (footnote 4 L1020, L1137-1139); f32 ADD results
+ *     are therefore equal to the exact sum only up to rounding;
+ *   - inputs are NaN-free (results unspecified otherwise).
+ *
+ * Conventions for every entry point:
+ *   - Ownership: the caller owns every buffer.  Pointers named in/out/ws are
+ *     DEVICE pointers on the current CUDA device; the library never allocates
+ *     or frees (allocation hoisting, L440-442).
+ *   - Freshness: outputs are fresh (L705-708, L537-539): an output range that
+ *     overlaps an input range is rejected with FS_ERR_ALIAS before any launch.
+ *   - Asynchrony: every call enqueues its kernels on `stream` (a cudaStream_t,
+ *     NULL = legacy default stream) and returns; results are valid in stream
+ *     order.
+ *   - Errors: FS_ERR_NULL / _SIZE / _UNSUPPORTED / _ALIAS / _WORKSPACE are
+ *     detected on the host before any launch (no side effects).  FS_ERR_CUDA
+ *     reports a failed launch.  Device-side precondition violations (a
+ *     stream_red key outside [0,k)) set an error word in the workspace that
+ *     fs_check_device_error() reports (L429-432: bounds checks).
+ *   - Workspace: `ws` is a device buffer of at least the size the matching
+ *     fs_*_workspace() query returns.  It must be zero-filled once before its
+ *     first use; every successful call leaves it ready for the next one.  One
+ *     workspace must not be used by two calls that may run concurrently.
+ *   - Empty inputs are legal: n = 0 reduces to 0(+) (index -1); seglen = 0
+ *     gives nseg copies of 0(+); a scan of nothing writes nothing.
+ *   - Layout of a [nseg][seglen] input: FS_ROW_MAJOR puts element (s, j) at
+ *     s*seglen + j; FS_COL_MAJOR at j*nseg + s (same type, other
+ *     representation, L1429-1434).
+ *   - ARGMIN outputs are zip/unzip split (L138-146): values in `out` (element
+ *     dtype), int64 indices in `out_idx`.  Indices are global positions for
+ *     redomap/scanomap and segment-local (0..seglen-1) for seg_*.
+ */
+#ifndef FUTSEG_H
+#define FUTSEG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum fs_dtype { FS_I32 = 0, FS_I64 = 1, FS_F32 = 2 } fs_dtype;
+
+typedef enum fs_op { FS_ADD = 0, FS_MIN = 1, FS_MAX = 2, FS_ARGMIN = 3, FS_VADD = 4 } fs_op;
+
+typedef enum fs_map_kind {
+    FS_MAP_ID = 0,     /* f x = x                                               */
+    FS_MAP_NN_DIST = 1 /* f (lat, lng) = sqrtf((lat-q0)^2 + (lng-q1)^2), every  */
+                       /* f32 operation separately rounded (no FMA contraction). */
+                       /* Rodinia NN (L1653-1656); inputs are SoA lat[], lng[]. */
+} fs_map_kind;
+
+typedef enum fs_layout { FS_ROW_MAJOR = 0, FS_COL_MAJOR = 1 } fs_layout;
+
+typedef enum fs_status {
+    FS_OK = 0,
+    FS_ERR_NULL = 1,        /* a required pointer is NULL                        */
+    FS_ERR_SIZE = 2,        /* negative size, or nseg*seglen / n*width overflows */
+    FS_ERR_UNSUPPORTED = 3, /* (op, dtype, map, primitive) not in the table      */
+    FS_ERR_ALIAS = 4,       /* an output range overlaps an input range           */
+    FS_ERR_WORKSPACE = 5,   /* ws is NULL or smaller than the query's answer     */
+    FS_ERR_CUDA = 6,        /* a CUDA launch or runtime call failed              */
+    FS_ERR_BOUNDS = 7       /* device-side precondition violation (stream_red)   */
+} fs_status;
+
+/* Operator descriptor.  width = k for FS_VADD (vectors of k elements), else 1. */
+typedef struct fs_opdesc {
+    int32_t op;    /* fs_op    */
+    int32_t dtype; /* fs_dtype */
+    int64_t width;
+} fs_opdesc;
+
+/* Map descriptor for the fused map stage of redomap / scanomap. */
+typedef struct fs_mapdesc {
+    int32_t kind;  /* fs_map_kind */
+    float q0, q1;  /* FS_MAP_NN_DIST query point (lat, lng); ignored otherwise */
+    int64_t ibase; /* global index of in0[0]: ARGMIN indices are ibase + position */
+                   /* (a shard of a larger array, see the multi-GPU layer); 0 */
+                   /* for a whole array.                                        */
+} fs_mapdesc;
+
+/* ---------------------------------------------------------------- workspace */
+/* Each query writes the workspace size (bytes) the matching call needs on the
+ * CURRENT device (it depends on the SM count) for the given sizes. */
+fs_status fs_redomap_workspace(fs_opdesc op, int64_t n, size_t *bytes);
+fs_status fs_scanomap_workspace(fs_opdesc op, int64_t n, size_t *bytes);
+fs_status fs_seg_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout,
+                                  size_t *bytes);
+fs_status fs_seg_scan_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout,
+                                size_t *bytes);
+fs_status fs_stream_red_workspace(int32_t dtype, int64_t n, int64_t w, int64_t k, size_t *bytes);
+
+/* ---------------------------------------------------------------- redomap */
+/* out = 0(+) (+) f(x_0) (+) ... (+) f(x_{n-1})       (fold, L240-241; F3 L1067)
+ *   op.op in {ADD, MIN, MAX, ARGMIN, VADD}; op.dtype in {I32, I64, F32}.
+ *   map.kind == FS_MAP_ID      : in0 = x, n elements of op.dtype (VADD: [n][width]
+ *                                row-major, n rows); in1 must be NULL.
+ *   map.kind == FS_MAP_NN_DIST : in0 = lat[n], in1 = lng[n] (f32); op.dtype must be
+ *                                F32 and op.op in {ADD, MIN, MAX, ARGMIN}.
+ *   out     : 1 element of op.dtype (VADD: width elements).
+ *   out_idx : ARGMIN only, 1 int64 (global index of the first minimum; -1 if n == 0).
+ * VADD(width) is the vectorised operator map(+) of Fig 4b; with op.op == VADD the
+ * result is the column sums of the [n][width] input (G5, L1313-1319). */
+fs_status fs_redomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *in1, int64_t n,
+                     void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
+
+/* ---------------------------------------------------------------- scanomap */
+/* out[i] = c (+) f(x_0) (+) ... (+) f(x_i)  for i < n   (scan L129-130; F5 L1071-1074)
+ *   Same op/map/input rules as fs_redomap, except op.op != VADD.
+ *   out: n elements of op.dtype; out_idx: ARGMIN only, n int64.
+ *   carry / carry_idx: optional DEVICE pointers to one element (and, for ARGMIN,
+ *   one int64 index) folded in front of the scan: c.  NULL means c = 0(+).
+ *   (Used to continue a scan across shards: F5's accumulator a.)
+ * Single-pass chained scan with decoupled look-back; the workspace holds the
+ * per-tile status words and is re-initialised by every call. */
+fs_status fs_scanomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *in1, int64_t n,
+                      void *out, int64_t *out_idx, const void *carry, const int64_t *carry_idx,
+                      void *ws, size_t ws_bytes, void *stream);
+
+/* ---------------------------------------------------------------- combine */
+/* out = parts[0] (+) parts[1] (+) ... (+) parts[P-1], in that order.
+ *   The final combine of per-chunk / per-GPU partial results (sFold's outer
+ *   (+), L259-260; stream_red's reduction across chunks, L1004-1006).
+ *   parts: P elements of op.dtype (VADD: [P][width]); part_idx: ARGMIN only, the
+ *   P partial indices (global positions).  P = 0 gives 0(+).  No workspace. */
+fs_status fs_combine(fs_opdesc op, const void *parts, const int64_t *part_idx, int64_t P, void *out,
+                     int64_t *out_idx, void *stream);
+
+/* ---------------------------------------------------------------- stream_red */
+/* The K-means centre update (Fig 4c; Sec. 2.4; L1649):
+ *   sums[c][j] = sum of vals[i][j] over i with keys[i] == c      (c < k, j < w)
+ *   counts[c]  = #{ i : keys[i] == c }
+ * computed as stream_red (map(+)): the input is split into chunks; each chunk
+ * folds its rows into a fresh zero [k][w] accumulator updated in place, and the
+ * chunk results are combined with the vectorised add (L526-531).
+ *   dtype in {I32, I64, F32} (vals and sums); keys are int32; counts int32 (wraps).
+ *   vals: [n][w] row-major; sums: [k][w]; counts may be NULL.
+ *   Outputs are overwritten (each chunk starts from the neutral zeros; no
+ *   user-supplied initial accumulator).  A key outside [0, k) is skipped and
+ *   raises the device error word (fs_check_device_error -> FS_ERR_BOUNDS). */
+fs_status fs_stream_red(int32_t dtype, const void *vals, const int32_t *keys, int64_t n, int64_t w,
+                        int64_t k, void *sums, int32_t *counts, void *ws, size_t ws_bytes,
+                        void *stream);
+
+/* ---------------------------------------------------------------- segmented */
+/* out[s] = reduce (+) 0(+) xss[s]  for s < nseg  (footnote 5; G5; Fig 11)
+ *   xss is the logical [nseg][seglen] array stored in `in` with `layout`.
+ *   op.op in {ADD, MIN, MAX, ARGMIN}; out: nseg elements; out_idx: ARGMIN only
+ *   (segment-local index).  The kernel is chosen by segment length
+ *   (fs_seg_reduce_regime). */
+fs_status fs_seg_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int32_t layout,
+                        void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
+
+/* out = map (scan (+) 0(+)) xss: the inclusive scan of every row; out has the
+ * shape and layout of in (footnote 5: a scan with a modified associative
+ * operator).  op.op in {ADD, MIN, MAX, ARGMIN}; out_idx: ARGMIN only (nseg*seglen
+ * int64, segment-local indices). */
+fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int32_t layout,
+                      void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
+
+/* ---------------------------------------------------------------- transpose */
+/* out[j][i] = in[i][j] for an in : [rows][cols] row-major array of dtype
+ * (4- or 8-byte elements); out : [cols][rows].  No workspace; no in-place. */
+fs_status fs_transpose_2d(int32_t dtype, const void *in, int64_t rows, int64_t cols, void *out,
+                          void *stream);
+
+/* ---------------------------------------------------------------- utilities */
+/* Synchronises `stream`, reads and clears the device error word of `ws`.
+ * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */
+fs_status fs_check_device_error(void *ws, void *stream);
+
+/* Regime the dispatcher picks for a segmented call on the current device:
+ *   0 = KG1 thread-per-segment over a shared-memory tile (short rows)
+ *   1 = KG2 warp per segment
+ *   2 = KG3 block per segment
+ *   3 = KG4 several blocks per segment, partials combined by the last block
+ *   4 = column kernel (FS_COL_MAJOR: thread per segment, coalesced rows)
+ *   5 = single-pass segmented look-back scan (fs_seg_scan, FS_ROW_MAJOR)
+ *   6 = empty input (neutral fill)
+ * Returns -1 for invalid arguments. */
+int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen,
+                      int32_t layout);
+
+/* Testing / sweep aid: force the seg_reduce regime (0..3 for FS_ROW_MAJOR) for
+ * subsequent calls in this process; -1 restores automatic selection.  Also
+ * settable with the environment variable FUTSEG_FORCE_REGIME. */
+fs_status fs_force_seg_regime(int32_t regime);
+
+const char *fs_status_string(fs_status s);
+const char *fs_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FUTSEG_H */

@@ -1,0 +1,376 @@
+// api.cu -- the extern "C" boundary of libfutseg (include/futseg.h).
+//
+// Host-side argument validation happens here, before any launch, so an error
+// status has no side effects (mirrors Futhark's hoisted dynamic shape and
+// bounds checks, L429-432).  The launchers it calls live in the per-kernel
+// translation units.
+#include <mutex>
+#include <stdlib.h>
+#include <unordered_map>
+
+#include "internal.cuh"
+
+namespace fs {
+
+// ------------------------------------------------------------ device queries
+int sm_count() {
+    static int cache[128] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 128) return 148;
+    if (cache[dev] == 0) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+        cache[dev] = v;
+    }
+    return cache[dev];
+}
+
+int max_blocks_per_sm(const void *kernel, int threads, size_t smem) {
+    static std::mutex mu;
+    static std::unordered_map<uint64_t, int> cache;
+    const uint64_t key = (uint64_t)(uintptr_t)kernel * 1000003ull ^ ((uint64_t)threads << 40) ^ (uint64_t)smem;
+    {
+        std::lock_guard<std::mutex> g(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+    }
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, threads, smem) != cudaSuccess || b <= 0) {
+        cudaGetLastError();
+        b = 1;
+    }
+    std::lock_guard<std::mutex> g(mu);
+    cache[key] = b;
+    return b;
+}
+
+static int g_forced_regime = -2;
+int forced_seg_regime() {
+    if (g_forced_regime == -2) {
+        const char *e = getenv("FUTSEG_FORCE_REGIME");
+        g_forced_regime = e ? atoi(e) : -1;
+    }
+    return g_forced_regime;
+}
+
+}  // namespace fs
+
+using namespace fs;
+
+namespace {
+
+bool valid_dtype(int dt) { return dt == FS_I32 || dt == FS_I64 || dt == FS_F32; }
+bool valid_scalar_op(int op) { return op == FS_ADD || op == FS_MIN || op == FS_MAX || op == FS_ARGMIN; }
+
+// op descriptor check; allow_vadd only for redomap
+fs_status check_op(const fs_opdesc &op, bool allow_vadd) {
+    if (!valid_dtype(op.dtype)) return FS_ERR_UNSUPPORTED;
+    if (op.op == FS_VADD) {
+        if (!allow_vadd) return FS_ERR_UNSUPPORTED;
+        if (op.width < 1) return FS_ERR_SIZE;
+        return FS_OK;
+    }
+    if (!valid_scalar_op(op.op)) return FS_ERR_UNSUPPORTED;
+    if (op.width > 1) return FS_ERR_UNSUPPORTED;
+    return FS_OK;
+}
+
+bool mul_overflows(int64_t a, int64_t b) { return a != 0 && b > INT64_MAX / a; }
+
+bool aligned_to(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+// do [a, a+na) and [b, b+nb) overlap?
+bool overlaps(const void *a, int64_t na, const void *b, int64_t nb) {
+    if (!a || !b || na <= 0 || nb <= 0) return false;
+    const uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+    return x < y + (uintptr_t)nb && y < x + (uintptr_t)na;
+}
+
+fs_status check_ws(void *ws, size_t have, size_t need) {
+    if (need == 0) return FS_OK;
+    if (!ws) return FS_ERR_WORKSPACE;
+    if (have < need) return FS_ERR_WORKSPACE;
+    if (!aligned_to(ws, 256)) return FS_ERR_WORKSPACE;
+    return FS_OK;
+}
+
+cudaStream_t S(void *stream) { return (cudaStream_t)stream; }
+
+#define FS_TRY(x)                           \
+    do {                                    \
+        fs_status _s = (x);                 \
+        if (_s != FS_OK) return _s;         \
+    } while (0)
+
+// map descriptor + inputs for redomap/scanomap
+fs_status check_map(const fs_opdesc &op, const fs_mapdesc &map, const void *in0, const void *in1, int64_t n) {
+    if (map.kind == FS_MAP_ID) {
+        if (in1) return FS_ERR_UNSUPPORTED;
+        if (n > 0 && !in0) return FS_ERR_NULL;
+        if (in0 && !aligned_to(in0, dtype_size(op.dtype))) return FS_ERR_UNSUPPORTED;
+        return FS_OK;
+    }
+    if (map.kind == FS_MAP_NN_DIST) {
+        if (op.dtype != FS_F32 || op.op == FS_VADD) return FS_ERR_UNSUPPORTED;
+        if (n > 0 && (!in0 || !in1)) return FS_ERR_NULL;
+        if ((in0 && !aligned_to(in0, 4)) || (in1 && !aligned_to(in1, 4))) return FS_ERR_UNSUPPORTED;
+        return FS_OK;
+    }
+    return FS_ERR_UNSUPPORTED;
+}
+
+int64_t in_bytes(const fs_opdesc &op, const fs_mapdesc &map, int64_t n) {
+    return n * (map.kind == FS_MAP_NN_DIST ? 4 : (int64_t)dtype_size(op.dtype) * (op.op == FS_VADD ? op.width : 1));
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *fs_version(void) { return "libfutseg 0.1 (sm_100a)"; }
+
+const char *fs_status_string(fs_status s) {
+    switch (s) {
+    case FS_OK: return "FS_OK";
+    case FS_ERR_NULL: return "FS_ERR_NULL: a required pointer is NULL";
+    case FS_ERR_SIZE: return "FS_ERR_SIZE: negative or overflowing size";
+    case FS_ERR_UNSUPPORTED: return "FS_ERR_UNSUPPORTED: (op, dtype, map, layout) not supported";
+    case FS_ERR_ALIAS: return "FS_ERR_ALIAS: output overlaps an input";
+    case FS_ERR_WORKSPACE: return "FS_ERR_WORKSPACE: workspace missing, misaligned or too small";
+    case FS_ERR_CUDA: return "FS_ERR_CUDA: CUDA launch or runtime error";
+    case FS_ERR_BOUNDS: return "FS_ERR_BOUNDS: device-side precondition violation (key out of range)";
+    }
+    return "unknown fs_status";
+}
+
+fs_status fs_force_seg_regime(int32_t regime) {
+    if (regime < -1 || regime > 3) return FS_ERR_UNSUPPORTED;
+    g_forced_regime = regime;
+    return FS_OK;
+}
+
+// ------------------------------------------------------------ workspace queries
+fs_status fs_redomap_workspace(fs_opdesc op, int64_t n, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    FS_TRY(check_op(op, true));
+    if (n < 0) return FS_ERR_SIZE;
+    if (op.op == FS_VADD) {
+        if (mul_overflows(n, op.width)) return FS_ERR_SIZE;
+        *bytes = colreduce_ws(FS_ADD, op.dtype, n, op.width);
+    } else {
+        *bytes = redomap_ws(op.op, op.dtype, n, false);
+    }
+    return FS_OK;
+}
+
+fs_status fs_scanomap_workspace(fs_opdesc op, int64_t n, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    FS_TRY(check_op(op, false));
+    if (n < 0) return FS_ERR_SIZE;
+    *bytes = scan_ws(op.op, op.dtype, n);
+    return FS_OK;
+}
+
+fs_status fs_seg_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    FS_TRY(check_op(op, false));
+    if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return FS_ERR_SIZE;
+    if (layout == FS_ROW_MAJOR) *bytes = seg_reduce_ws(op.op, op.dtype, nseg, seglen);
+    else if (layout == FS_COL_MAJOR) *bytes = colreduce_ws(op.op, op.dtype, seglen, nseg);
+    else return FS_ERR_UNSUPPORTED;
+    return FS_OK;
+}
+
+fs_status fs_seg_scan_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    FS_TRY(check_op(op, false));
+    if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return FS_ERR_SIZE;
+    if (layout == FS_ROW_MAJOR) *bytes = scan_ws(op.op, op.dtype, nseg * seglen);
+    else if (layout == FS_COL_MAJOR) *bytes = colscan_ws(op.op, op.dtype, seglen, nseg);
+    else return FS_ERR_UNSUPPORTED;
+    return FS_OK;
+}
+
+fs_status fs_stream_red_workspace(int32_t dtype, int64_t n, int64_t w, int64_t k, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (n < 0 || w < 0 || k < 0 || mul_overflows(n, w) || mul_overflows(k, w)) return FS_ERR_SIZE;
+    *bytes = stream_red_ws(dtype, n, w, k);
+    return FS_OK;
+}
+
+// ------------------------------------------------------------ redomap
+fs_status fs_redomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *in1, int64_t n, void *out,
+                     int64_t *out_idx, void *ws, size_t ws_bytes, void *stream) {
+    FS_TRY(check_op(op, true));
+    if (n < 0) return FS_ERR_SIZE;
+    if (op.op == FS_VADD && mul_overflows(n, op.width * (int64_t)dtype_size(op.dtype))) return FS_ERR_SIZE;
+    FS_TRY(check_map(op, map, in0, in1, n));
+    if (!out) return FS_ERR_NULL;
+    if (op.op == FS_ARGMIN && !out_idx) return FS_ERR_NULL;
+    if (!aligned_to(out, dtype_size(op.dtype)) || (out_idx && !aligned_to(out_idx, 8))) return FS_ERR_UNSUPPORTED;
+    const int64_t ib = in_bytes(op, map, n);
+    const int64_t ob = (op.op == FS_VADD ? op.width : 1) * (int64_t)dtype_size(op.dtype);
+    if (overlaps(out, ob, in0, ib) || overlaps(out, ob, in1, ib) ||
+        (op.op == FS_ARGMIN && (overlaps(out_idx, 8, in0, ib) || overlaps(out_idx, 8, in1, ib) ||
+                                overlaps(out_idx, 8, out, ob))))
+        return FS_ERR_ALIAS;
+    size_t need = 0;
+    FS_TRY(fs_redomap_workspace(op, n, &need));
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    if (op.op == FS_VADD) {
+        if (n == 0) return fill_neutral_run(FS_ADD, op.dtype, op.width, out, nullptr, S(stream));
+        return colreduce_run(FS_ADD, op.dtype, in0, n, op.width, out, nullptr, ws, S(stream));
+    }
+    return redomap_run(op.op, op.dtype, map, in0, in1, n, out, op.op == FS_ARGMIN ? out_idx : nullptr, ws,
+                       S(stream));
+}
+
+// ------------------------------------------------------------ scanomap
+fs_status fs_scanomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *in1, int64_t n, void *out,
+                      int64_t *out_idx, const void *carry, const int64_t *carry_idx, void *ws, size_t ws_bytes,
+                      void *stream) {
+    FS_TRY(check_op(op, false));
+    if (n < 0) return FS_ERR_SIZE;
+    FS_TRY(check_map(op, map, in0, in1, n));
+    if (n > 0 && !out) return FS_ERR_NULL;
+    if (n > 0 && op.op == FS_ARGMIN && !out_idx) return FS_ERR_NULL;
+    if (carry && op.op == FS_ARGMIN && !carry_idx) return FS_ERR_NULL;
+    if ((out && !aligned_to(out, dtype_size(op.dtype))) || (out_idx && !aligned_to(out_idx, 8)))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t ib = in_bytes(op, map, n);
+    const int64_t ob = n * (int64_t)dtype_size(op.dtype);
+    if (overlaps(out, ob, in0, ib) || overlaps(out, ob, in1, ib) ||
+        (op.op == FS_ARGMIN && (overlaps(out_idx, 8 * n, in0, ib) || overlaps(out_idx, 8 * n, in1, ib) ||
+                                overlaps(out_idx, 8 * n, out, ob))))
+        return FS_ERR_ALIAS;
+    size_t need = 0;
+    FS_TRY(fs_scanomap_workspace(op, n, &need));
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    if (n == 0) return FS_OK;
+    return scan_run(op.op, op.dtype, map, in0, in1, n, n, out, op.op == FS_ARGMIN ? out_idx : nullptr, carry,
+                    op.op == FS_ARGMIN ? carry_idx : nullptr, ws, S(stream));
+}
+
+// ------------------------------------------------------------ combine
+fs_status fs_combine(fs_opdesc op, const void *parts, const int64_t *part_idx, int64_t P, void *out,
+                     int64_t *out_idx, void *stream) {
+    FS_TRY(check_op(op, true));
+    if (P < 0) return FS_ERR_SIZE;
+    if (P > 0 && !parts) return FS_ERR_NULL;
+    if (!out) return FS_ERR_NULL;
+    if (op.op == FS_ARGMIN && (!out_idx || (P > 0 && !part_idx))) return FS_ERR_NULL;
+    const int64_t w = op.op == FS_VADD ? op.width : 1;
+    if (mul_overflows(P, w)) return FS_ERR_SIZE;
+    const int64_t pb = P * w * (int64_t)dtype_size(op.dtype), ob = w * (int64_t)dtype_size(op.dtype);
+    if (overlaps(out, ob, parts, pb) || overlaps(out, ob, part_idx, 8 * P)) return FS_ERR_ALIAS;
+    return combine_run(op.op, op.dtype, w, parts, part_idx, P, out, op.op == FS_ARGMIN ? out_idx : nullptr,
+                       S(stream));
+}
+
+// ------------------------------------------------------------ stream_red
+fs_status fs_stream_red(int32_t dtype, const void *vals, const int32_t *keys, int64_t n, int64_t w, int64_t k,
+                        void *sums, int32_t *counts, void *ws, size_t ws_bytes, void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (n < 0 || w < 0 || k < 0 || mul_overflows(n, w) || mul_overflows(k, w)) return FS_ERR_SIZE;
+    if (n > 0 && (!keys || (w > 0 && !vals))) return FS_ERR_NULL;
+    if (k > 0 && w > 0 && !sums) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype);
+    if ((vals && !aligned_to(vals, es)) || (sums && !aligned_to(sums, es)) || (keys && !aligned_to(keys, 4)) ||
+        (counts && !aligned_to(counts, 4)))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t vb = n * w * es, kb = 4 * n, sb = k * w * es, cb = 4 * k;
+    if (overlaps(sums, sb, vals, vb) || overlaps(sums, sb, keys, kb) || overlaps(counts, cb, vals, vb) ||
+        overlaps(counts, cb, keys, kb) || overlaps(counts, cb, sums, sb))
+        return FS_ERR_ALIAS;
+    size_t need = 0;
+    FS_TRY(fs_stream_red_workspace(dtype, n, w, k, &need));
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    if (k == 0) return FS_OK;
+    return stream_red_run(dtype, vals, keys, n, w, k, sums, counts, ws, S(stream));
+}
+
+// ------------------------------------------------------------ segmented
+static fs_status seg_common(const fs_opdesc &op, const void *in, int64_t nseg, int64_t seglen, int32_t layout,
+                            void *out, int64_t *out_idx, int64_t out_elems) {
+    FS_TRY(check_op(op, false));
+    if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen) ||
+        mul_overflows(nseg * seglen, (int64_t)sizeof(int64_t)))
+        return FS_ERR_SIZE;
+    if (layout != FS_ROW_MAJOR && layout != FS_COL_MAJOR) return FS_ERR_UNSUPPORTED;
+    if (nseg * seglen > 0 && !in) return FS_ERR_NULL;
+    if (out_elems > 0 && !out) return FS_ERR_NULL;
+    if (out_elems > 0 && op.op == FS_ARGMIN && !out_idx) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(op.dtype);
+    if ((in && !aligned_to(in, es)) || (out && !aligned_to(out, es)) || (out_idx && !aligned_to(out_idx, 8)))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t ib = nseg * seglen * es, ob = out_elems * es;
+    if (overlaps(out, ob, in, ib) ||
+        (op.op == FS_ARGMIN && (overlaps(out_idx, 8 * out_elems, in, ib) || overlaps(out_idx, 8 * out_elems, out, ob))))
+        return FS_ERR_ALIAS;
+    return FS_OK;
+}
+
+fs_status fs_seg_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int32_t layout, void *out,
+                        int64_t *out_idx, void *ws, size_t ws_bytes, void *stream) {
+    FS_TRY(seg_common(op, in, nseg, seglen, layout, out, out_idx, nseg));
+    size_t need = 0;
+    FS_TRY(fs_seg_reduce_workspace(op, nseg, seglen, layout, &need));
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
+    if (nseg == 0) return FS_OK;
+    if (seglen == 0) return fill_neutral_run(op.op, op.dtype, nseg, out, oi, S(stream));
+    if (layout == FS_COL_MAJOR) return colreduce_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
+    return seg_reduce_run(op.op, op.dtype, in, nseg, seglen, out, oi, ws, S(stream));
+}
+
+fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int32_t layout, void *out,
+                      int64_t *out_idx, void *ws, size_t ws_bytes, void *stream) {
+    FS_TRY(seg_common(op, in, nseg, seglen, layout, out, out_idx, nseg * seglen));
+    size_t need = 0;
+    FS_TRY(fs_seg_scan_workspace(op, nseg, seglen, layout, &need));
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
+    if (nseg * seglen == 0) return FS_OK;
+    if (layout == FS_COL_MAJOR) return colscan_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
+    const fs_mapdesc id = {FS_MAP_ID, 0.f, 0.f};
+    return scan_run(op.op, op.dtype, id, in, nullptr, nseg * seglen, seglen, out, oi, nullptr, nullptr, ws,
+                    S(stream));
+}
+
+// ------------------------------------------------------------ transpose
+fs_status fs_transpose_2d(int32_t dtype, const void *in, int64_t rows, int64_t cols, void *out, void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (rows < 0 || cols < 0 || mul_overflows(rows, cols) || mul_overflows(rows * cols, 8)) return FS_ERR_SIZE;
+    if (rows * cols == 0) return FS_OK;
+    if (!in || !out) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype);
+    if (!aligned_to(in, es) || !aligned_to(out, es)) return FS_ERR_UNSUPPORTED;
+    if (overlaps(out, rows * cols * es, in, rows * cols * es)) return FS_ERR_ALIAS;
+    return transpose_run(dtype, in, rows, cols, out, S(stream));
+}
+
+// ------------------------------------------------------------ utilities
+fs_status fs_check_device_error(void *ws, void *stream) {
+    if (!ws) return FS_ERR_NULL;
+    if (cudaStreamSynchronize(S(stream)) != cudaSuccess) return FS_ERR_CUDA;
+    unsigned err = 0;
+    unsigned *p = (unsigned *)((char *)ws + kWsErr);
+    if (cudaMemcpy(&err, p, sizeof(err), cudaMemcpyDeviceToHost) != cudaSuccess) return FS_ERR_CUDA;
+    if (err) {
+        if (cudaMemset(p, 0, sizeof(unsigned)) != cudaSuccess) return FS_ERR_CUDA;
+        return FS_ERR_BOUNDS;
+    }
+    return FS_OK;
+}
+
+int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout) {
+    if (check_op(op, false) != FS_OK || nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return -1;
+    if (layout != FS_ROW_MAJOR && layout != FS_COL_MAJOR) return -1;
+    if (nseg == 0 || seglen == 0) return 6;
+    if (layout == FS_COL_MAJOR) return 4;
+    if (prim_is_scan) return 5;
+    return seg_reduce_regime(op.op, op.dtype, nseg, seglen);
+}
+
+}  // extern "C"

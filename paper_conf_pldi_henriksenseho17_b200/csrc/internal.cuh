@@ -1,0 +1,84 @@
+// internal.cuh -- host-side helpers shared by the kernel translation units and
+// the C ABI (api.cu): device properties, occupancy-derived grid sizes, the
+// (op, dtype) template dispatcher, and the per-primitive launchers.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include "common.cuh"
+
+namespace fs {
+
+int sm_count();  // SMs of the current device (cached per device)
+int max_blocks_per_sm(const void *kernel, int threads, size_t dyn_smem);  // cached
+inline int resident_blocks(const void *kernel, int threads, size_t smem = 0) {
+    return sm_count() * max_blocks_per_sm(kernel, threads, smem);
+}
+int forced_seg_regime();  // -1 = automatic
+
+inline fs_status launch_status() {
+    return cudaGetLastError() == cudaSuccess ? FS_OK : FS_ERR_CUDA;
+}
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// (op, dtype) -> F<OP, T>::run(args...).  ops limited to ADD/MIN/MAX/ARGMIN.
+template <template <int, typename> class F, typename T, typename... A>
+fs_status dispatch_op(int op, A... a) {
+    switch (op) {
+    case FS_ADD: return F<kAdd, T>::run(a...);
+    case FS_MIN: return F<kMin, T>::run(a...);
+    case FS_MAX: return F<kMax, T>::run(a...);
+    case FS_ARGMIN: return F<kArgmin, T>::run(a...);
+    }
+    return FS_ERR_UNSUPPORTED;
+}
+template <template <int, typename> class F, typename... A>
+fs_status dispatch(int op, int dt, A... a) {
+    switch (dt) {
+    case FS_I32: return dispatch_op<F, int32_t>(op, a...);
+    case FS_I64: return dispatch_op<F, int64_t>(op, a...);
+    case FS_F32: return dispatch_op<F, float>(op, a...);
+    }
+    return FS_ERR_UNSUPPORTED;
+}
+
+inline size_t dtype_size(int dt) { return dt == FS_I64 ? 8 : 4; }
+// bytes of one accumulator V for (op, dt)
+inline size_t acc_size(int op, int dt) { return op == FS_ARGMIN ? 16 : dtype_size(dt); }
+
+// ---- launchers (one per translation unit); arguments already validated ----
+// redomap.cu
+size_t redomap_ws(int op, int dt, int64_t n, bool nn);
+fs_status redomap_run(int op, int dt, const fs_mapdesc &map, const void *in0, const void *in1, int64_t n,
+                      void *out, int64_t *out_idx, void *ws, cudaStream_t st);
+fs_status combine_run(int op, int dt, int64_t width, const void *parts, const int64_t *part_idx, int64_t P,
+                      void *out, int64_t *out_idx, cudaStream_t st);
+// colreduce.cu  ([m][w] row-major -> [w], any op; index = row)
+size_t colreduce_ws(int op, int dt, int64_t m, int64_t w);
+fs_status colreduce_run(int op, int dt, const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx,
+                        void *ws, cudaStream_t st);
+// seg_reduce.cu (row-major regimes)
+int seg_reduce_regime(int op, int dt, int64_t nseg, int64_t seglen);
+size_t seg_reduce_ws(int op, int dt, int64_t nseg, int64_t seglen);
+fs_status seg_reduce_run(int op, int dt, const void *in, int64_t nseg, int64_t seglen, void *out,
+                         int64_t *out_idx, void *ws, cudaStream_t st);
+fs_status fill_neutral_run(int op, int dt, int64_t count, void *out, int64_t *out_idx, cudaStream_t st);
+// scan.cu
+size_t scan_ws(int op, int dt, int64_t n);
+fs_status scan_run(int op, int dt, const fs_mapdesc &map, const void *in0, const void *in1, int64_t n,
+                   int64_t seglen, void *out, int64_t *out_idx, const void *carry, const int64_t *carry_idx,
+                   void *ws, cudaStream_t st);
+size_t colscan_ws(int op, int dt, int64_t m, int64_t w);
+fs_status colscan_run(int op, int dt, const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx,
+                      void *ws, cudaStream_t st);
+// stream_red.cu
+size_t stream_red_ws(int dt, int64_t n, int64_t w, int64_t k);
+fs_status stream_red_run(int dt, const void *vals, const int32_t *keys, int64_t n, int64_t w, int64_t k,
+                         void *sums, int32_t *counts, void *ws, cudaStream_t st);
+// transpose.cu
+fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
+
+}  // namespace fs

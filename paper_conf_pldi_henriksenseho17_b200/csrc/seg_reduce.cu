@@ -1,0 +1,334 @@
+// seg_reduce.cu -- segmented reduction over a regular FS_ROW_MAJOR
+// [nseg][seglen] array: out[s] = reduce (+) 0(+) xss[s]   (footnote 5,
+// L1230-1233: a map nest ending in a reduce; Fig 11's map-map-reduce nest).
+//
+// The paper's flattening has "no size that fits all" and proposes choosing
+// between code versions at run time (L1411-1418).  This file is that choice,
+// by segment length L (thresholds in seg_reduce_regime, calibrated by the
+// seglen sweep in bench/ncu):
+//   KG1  L small  : a CTA stages a tile of whole segments in shared memory
+//                   with coalesced 16-byte loads, then groups of G lanes
+//                   (G ~ L/4, a power of two) reduce one segment each.
+//                   Shared memory is padded every 32 (4-byte) / 16 (8-byte)
+//                   elements so strided per-segment reads do not conflict.
+//   KG2  L medium : one warp per segment, 16-byte loads straight from HBM.
+//   KG3  L large, many segments : one CTA per segment.
+//   KG4  L large, few segments  : C CTAs per segment; each writes a partial
+//                   and the last to arrive (per-segment ticket) combines the
+//                   C partials in chunk order (the "second pass", fused).
+#include "internal.cuh"
+
+namespace fs {
+
+constexpr int kSegThreads = 256;
+constexpr int kTileBytes = 32768;  // KG1 staged tile (before padding)
+
+template <typename T> __device__ __forceinline__ int pad_pos(int e) {
+    return sizeof(T) == 4 ? e + (e >> 5) : e + (e >> 4);
+}
+template <typename T> __host__ __device__ constexpr int tile_elems() { return kTileBytes / (int)sizeof(T); }
+template <typename T> __host__ __device__ constexpr int tile_smem_bytes() {
+    return (tile_elems<T>() + tile_elems<T>() / (sizeof(T) == 4 ? 32 : 16) + 4) * (int)sizeof(T);
+}
+
+// ---------------------------------------------------------------- KG1
+template <int OP, typename T, int NT, int G>
+__global__ void __launch_bounds__(NT)
+seg_tile_kernel(const T *__restrict__ x, int64_t nseg, int L, int tile_segs, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    constexpr int U = 8;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T *sm = reinterpret_cast<T *>(smem_raw);
+    const int t = threadIdx.x;
+    const bool vec_ok = (((uintptr_t)x & 15) == 0);  // host guarantees tile_segs*L*sizeof(T) % 16 == 0
+    const int64_t ntiles = (nseg + tile_segs - 1) / tile_segs;
+    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int64_t seg0 = tile * tile_segs;
+        const int segs = (int)((nseg - seg0) < tile_segs ? (nseg - seg0) : tile_segs);
+        const int ecount = segs * L;
+        const T *src = x + seg0 * (int64_t)L;
+        int done = 0;
+        if (vec_ok) {
+            const int nv = ecount / VEC;
+            const int4 *sv = reinterpret_cast<const int4 *>(src);
+            for (int v0 = t; v0 < nv; v0 += NT * U) {
+                int4 r[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (v0 + u * NT < nv) r[u] = ldg16(sv + v0 + u * NT);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (v0 + u * NT < nv) {
+                        const Vec16<T> e = as_vec<T>(r[u]);
+                        const int b = (v0 + u * NT) * VEC;
+#pragma unroll
+                        for (int k = 0; k < VEC; ++k) sm[pad_pos<T>(b + k)] = e.e[k];
+                    }
+            }
+            done = nv * VEC;
+        }
+        for (int e = done + t; e < ecount; e += NT) sm[pad_pos<T>(e)] = __ldg(src + e);
+        __syncthreads();
+        // reduce: group g of G lanes takes segment (base + g)
+        constexpr int NG = NT / G;
+        const int lg = t % G;
+        for (int base = 0; base < segs; base += NG) {
+            const int sl = base + t / G;
+            V a = O::id();
+            if (sl < segs) {
+                const int off = sl * L;
+                for (int j = lg; j < L; j += G) a = O::fold(a, sm[pad_pos<T>(off + j)], j);
+            }
+            a = group_reduce<O, G>(a);
+            if (lg == 0 && sl < segs) store_out<O>(out, out_idx, seg0 + sl, a);
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------- KG2
+template <int OP, typename T, int NT, int U>
+__global__ void __launch_bounds__(NT)
+seg_warp_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * NT + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * NT) >> 5;
+    for (int64_t s = gw; s < nseg; s += nw) {
+        const T *p = x + s * L;
+        int64_t head = (int64_t)(((16 - ((uintptr_t)p & 15)) & 15) / sizeof(T));
+        if (head > L) head = L;
+        const int64_t nvec = (L - head) / VEC, tail0 = head + nvec * VEC;
+        const int4 *pv = reinterpret_cast<const int4 *>(p + head);
+        V a = O::id();
+        if (lane < head) a = O::fold(a, __ldg(p + lane), lane);
+        int64_t v = lane;
+        for (; v + (U - 1) * 32 < nvec; v += U * 32) {
+            int4 r[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) r[u] = ldg16(pv + v + u * 32);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const Vec16<T> e = as_vec<T>(r[u]);
+                const int64_t b = head + (v + u * 32) * VEC;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], b + k);
+            }
+        }
+        for (; v < nvec; v += 32) {
+            const Vec16<T> e = as_vec<T>(ldg16(pv + v));
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], head + v * VEC + k);
+        }
+        if (lane < L - tail0) a = O::fold(a, __ldg(p + tail0 + lane), tail0 + lane);
+        a = group_reduce<O>(a);
+        if (lane == 0) store_out<O>(out, out_idx, s, a);
+    }
+}
+
+// ---------------------------------------------------------------- KG3 / KG4
+template <int OP, typename T, int NT, int U>
+__global__ void __launch_bounds__(NT)
+seg_block_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, int64_t C, int64_t CS,
+                 typename Op<OP, T>::V *partials, unsigned *tickets, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    __shared__ V sm[32];
+    __shared__ bool last;
+    const int t = threadIdx.x;
+    const int64_t items = nseg * C;
+    for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+        const int64_t s = it / C, c = it - s * C;
+        const int64_t j0 = c * CS;
+        const int64_t j1 = j0 + CS < L ? j0 + CS : L;
+        const T *p = x + s * L + j0;
+        const int64_t len = j1 > j0 ? j1 - j0 : 0;
+        int64_t head = (int64_t)(((16 - ((uintptr_t)p & 15)) & 15) / sizeof(T));
+        if (head > len) head = len;
+        const int64_t nvec = (len - head) / VEC, tail0 = head + nvec * VEC;
+        const int4 *pv = reinterpret_cast<const int4 *>(p + head);
+        V a = O::id();
+        if (t < head) a = O::fold(a, __ldg(p + t), j0 + t);
+        int64_t v = t;
+        for (; v + (int64_t)(U - 1) * NT < nvec; v += (int64_t)U * NT) {
+            int4 r[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) r[u] = ldg16(pv + v + u * NT);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const Vec16<T> e = as_vec<T>(r[u]);
+                const int64_t b = j0 + head + (v + u * NT) * VEC;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], b + k);
+            }
+        }
+        for (; v < nvec; v += NT) {
+            const Vec16<T> e = as_vec<T>(ldg16(pv + v));
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], j0 + head + v * VEC + k);
+        }
+        if (t < len - tail0) a = O::fold(a, __ldg(p + tail0 + t), j0 + tail0 + t);
+        a = block_reduce<O, NT>(a, sm);
+        if (C == 1) {
+            if (t == 0) store_out<O>(out, out_idx, s, a);
+            continue;
+        }
+        if (t == 0) {
+            st_cg(partials + it, a);
+            __threadfence();
+            last = atomicAdd(tickets + s, 1u) == (unsigned)(C - 1);
+        }
+        __syncthreads();
+        if (last) {
+            __threadfence();
+            V b = O::id();
+            for (int64_t q = t; q < C; q += NT) b = O::comb(b, ld_cg(partials + s * C + q));
+            b = block_reduce<O, NT>(b, sm);
+            if (t == 0) {
+                store_out<O>(out, out_idx, s, b);
+                atomicExch(tickets + s, 0u);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+template <int OP, typename T>
+__global__ void fill_neutral_kernel(int64_t count, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < count; k += (int64_t)gridDim.x * blockDim.x)
+        store_out<O>(out, out_idx, k, O::id());
+}
+
+// ---------------------------------------------------------------- host
+constexpr int64_t kWarpMaxL = 8192;    // KG2 upper bound (calibrated)
+constexpr int64_t kMinChunk = 16384;   // KG4 smallest chunk (elements)
+
+template <typename T> static int kg1_max_len() { return tile_elems<T>() / 4; }
+
+int seg_reduce_regime(int op, int dt, int64_t nseg, int64_t L) {
+    (void)op;
+    if (nseg == 0 || L == 0) return 6;
+    const int kg1max = dt == FS_I64 ? kg1_max_len<int64_t>() : kg1_max_len<int32_t>();
+    const int forced = forced_seg_regime();
+    if (forced >= 0 && forced <= 3) {
+        if (forced == 0 && L > kg1max) return 1;
+        return forced;
+    }
+    if (L <= 64) return 0;
+    if (L <= kWarpMaxL) return 1;
+    const int64_t resident = (int64_t)sm_count() * 8;
+    return nseg >= 2 * resident ? 2 : 3;
+}
+
+struct BlockPlan {
+    int64_t C, CS, items, grid;
+};
+static BlockPlan block_plan(int dt, int64_t nseg, int64_t L, int regime) {
+    BlockPlan p;
+    const int64_t resident = (int64_t)sm_count() * 8;
+    const int64_t VEC = 16 / (int64_t)dtype_size(dt);
+    p.C = 1;
+    if (regime == 3) {
+        const int64_t want = ceil_div(4 * resident, nseg);
+        const int64_t maxc = ceil_div(L, kMinChunk);
+        p.C = want < maxc ? want : maxc;
+        if (p.C < 1 || nseg > kWsMaxTickets) p.C = 1;  // per-segment tickets live in the ws header
+    }
+    p.CS = ceil_div(ceil_div(L, p.C), VEC) * VEC;
+    p.C = ceil_div(L, p.CS);
+    p.items = nseg * p.C;
+    p.grid = p.items < resident ? p.items : resident;
+    return p;
+}
+
+template <int OP, typename T> struct SegRun {
+    static fs_status run(int regime, const void *in, int64_t nseg, int64_t L, void *out, int64_t *out_idx,
+                         void *ws, cudaStream_t st) {
+        using V = typename Op<OP, T>::V;
+        const T *x = (const T *)in;
+        if (regime == 0) {
+            const int maxe = tile_elems<T>();
+            int tile_segs = maxe / (int)L;
+            tile_segs &= ~3;  // L <= tile_elems/4: every tile start stays 16-byte aligned
+            const int64_t ntiles = ceil_div(nseg, tile_segs);
+            const int smem = tile_smem_bytes<T>();
+            void (*k)(const T *, int64_t, int, int, T *, int64_t *);
+            if (L < 8) k = seg_tile_kernel<OP, T, kSegThreads, 1>;
+            else if (L < 16) k = seg_tile_kernel<OP, T, kSegThreads, 2>;
+            else if (L < 32) k = seg_tile_kernel<OP, T, kSegThreads, 4>;
+            else if (L < 64) k = seg_tile_kernel<OP, T, kSegThreads, 8>;
+            else if (L < 128) k = seg_tile_kernel<OP, T, kSegThreads, 16>;
+            else k = seg_tile_kernel<OP, T, kSegThreads, 32>;
+            static bool attr_set = false;
+            if (!attr_set) {
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                cudaFuncSetAttribute((const void *)seg_tile_kernel<OP, T, kSegThreads, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                attr_set = true;
+            }
+            const int64_t cap = resident_blocks((const void *)k, kSegThreads, smem);
+            const int64_t grid = ntiles < cap ? ntiles : cap;
+            k<<<(unsigned)grid, kSegThreads, smem, st>>>(x, nseg, (int)L, tile_segs, (T *)out, out_idx);
+            return launch_status();
+        }
+        if (regime == 1) {
+            const void *k = (const void *)seg_warp_kernel<OP, T, kSegThreads, 4>;
+            const int64_t cap = resident_blocks(k, kSegThreads);
+            int64_t grid = ceil_div(nseg, kSegThreads / 32);
+            grid = grid < cap ? grid : cap;
+            seg_warp_kernel<OP, T, kSegThreads, 4><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, L, (T *)out, out_idx);
+            return launch_status();
+        }
+        const BlockPlan p = block_plan(sizeof(T) == 8 ? FS_I64 : FS_I32, nseg, L, regime);
+        char *w = (char *)ws;
+        V *parts = (V *)(w + kWsHeader);
+        unsigned *tickets = (unsigned *)(w + kWsTickets);
+        seg_block_kernel<OP, T, kSegThreads, 4><<<(unsigned)p.grid, kSegThreads, 0, st>>>(
+            x, nseg, L, p.C, p.CS, parts, tickets, (T *)out, out_idx);
+        return launch_status();
+    }
+};
+
+template <int OP, typename T> struct FillRun {
+    static fs_status run(int64_t count, void *out, int64_t *out_idx, cudaStream_t st) {
+        if (count <= 0) return FS_OK;
+        int64_t grid = ceil_div(count, 256);
+        grid = grid > 4096 ? 4096 : grid;
+        fill_neutral_kernel<OP, T><<<(unsigned)grid, 256, 0, st>>>(count, (T *)out, out_idx);
+        return launch_status();
+    }
+};
+
+size_t seg_reduce_ws(int op, int dt, int64_t nseg, int64_t L) {
+    const int r = seg_reduce_regime(op, dt, nseg, L);
+    size_t body = 0;
+    // KG3/KG4 may be forced for any length: size for the block plan of regime 3
+    if (nseg > 0 && L > 0) {
+        const BlockPlan p = block_plan(dt, nseg, L, 3);
+        body = align_up((size_t)(p.C > 1 ? p.items : 0) * acc_size(op, dt), 256);
+    }
+    (void)r;
+    return kWsHeader + body;
+}
+
+fs_status seg_reduce_run(int op, int dt, const void *in, int64_t nseg, int64_t L, void *out, int64_t *out_idx,
+                         void *ws, cudaStream_t st) {
+    const int regime = seg_reduce_regime(op, dt, nseg, L);
+    if (regime == 6) return fill_neutral_run(op, dt, nseg, out, out_idx, st);
+    return dispatch<SegRun>(op, dt, regime, in, nseg, L, out, out_idx, ws, st);
+}
+
+fs_status fill_neutral_run(int op, int dt, int64_t count, void *out, int64_t *out_idx, cudaStream_t st) {
+    return dispatch<FillRun>(op, dt, count, out, out_idx, st);
+}
+
+}  // namespace fs

@@ -1,0 +1,378 @@
+"""GPU parity: every libfutseg primitive (through the C ABI, via the binding)
+against the sequential CPU oracle on the same seeded inputs.
+
+Bar (BASELINE.json north_star):
+  * integers, indices, argmin (value and index), min/max: bit-exact;
+  * f32 add: |gpu - oracle_f64| <= 1e-4 * sum|x| (per output; for non-negative
+    data this is the 1e-4 relative bound), every scan position checked.
+Sizes span several tiles and a ragged tail; edge cases: empty, one element,
+misaligned (offset) pointers, ties, every segmented regime forced.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads
+
+pytestmark = pytest.mark.gpu
+
+DTYPES = [np.int32, np.int64, np.float32]
+OPS = ["add", "min", "max", "argmin"]
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module")
+def fs():
+    import paper_conf_pldi_henriksenseho17_b200 as m
+    return m
+
+
+def cu(a, offset=0):
+    """numpy -> CUDA tensor; offset > 0 returns a view starting `offset` elements in (misaligned)."""
+    a = np.ascontiguousarray(a)
+    if offset:
+        pad = np.zeros(offset, a.dtype)
+        t = torch.from_numpy(np.concatenate([pad, a.reshape(-1)])).cuda()
+        return t[offset:].view(a.shape) if a.ndim > 1 else t[offset:]
+    return torch.from_numpy(a).cuda()
+
+
+def host(t):
+    return t.detach().cpu().numpy()
+
+
+def assert_reduced(got, want, op, absx_sum=None, where=""):
+    """got: GPU result (tensor or (v, i)); want: oracle result; absx_sum: oracle sum of |x| (f32 add)."""
+    if op == "argmin":
+        gv, gi = host(got[0]), host(got[1])
+        wv, wi = want
+        np.testing.assert_array_equal(gi, wi, err_msg=f"argmin index {where}")
+        np.testing.assert_array_equal(gv, wv, err_msg=f"argmin value {where}")
+        return
+    g = host(got)
+    w = np.asarray(want)
+    if op == "add" and w.dtype == np.float64:
+        bound = TOL * np.asarray(absx_sum, np.float64) + 1e-30
+        err = np.abs(g.astype(np.float64) - w)
+        assert np.all(err <= bound), f"f32 add {where}: max err {err.max()} bound {np.min(bound)}"
+    else:
+        np.testing.assert_array_equal(g, w, err_msg=f"{op} {where}")
+
+
+# ------------------------------------------------------------------ redomap
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("op", OPS)
+@pytest.mark.parametrize("n,offset", [(0, 0), (1, 0), (3, 1), (1000, 0), (65537, 3), (1 << 20, 0), (3_000_017, 1)])
+def test_redomap(fs, dt, op, n, offset):
+    x = workloads.mixed(n, 100 + n, dt)
+    if n > 10 and op == "argmin":
+        x[n // 3] = x[n // 2] = x.min()  # tie: the first occurrence must win
+    got = fs.redomap(cu(x, offset), op)
+    want = oracle.reduce(x, op)
+    asum = oracle.reduce(np.abs(x), "add") if op == "add" and dt == np.float32 else None
+    assert_reduced(got, want, op, asum, f"n={n} off={offset}")
+    if op == "argmin" and n == 0:
+        assert int(host(got[1])) == -1
+
+
+def test_redomap_c1_full_range_bitexact(fs):
+    """BASELINE configs[0]: i32 sum over 2^20 full-range values (wraps), bit-exact."""
+    x = workloads.c1()
+    assert int(host(fs.redomap(cu(x), "add"))) == int(oracle.reduce(x, "add"))
+    xs = workloads.c1(small_range=True)
+    assert int(host(fs.redomap(cu(xs), "add"))) == int(oracle.reduce(xs, "add"))
+    for op in ("min", "max"):
+        assert int(host(fs.redomap(cu(x), op))) == int(oracle.reduce(x, op))
+
+
+@pytest.mark.parametrize("op", OPS)
+def test_redomap_nn_c2(fs, op):
+    """BASELINE configs[1]: Rodinia NN argmin over 855,280 (lat, lng) f32 records, duplicated 20x."""
+    lat, lng, q = workloads.c2_nn()
+    got = fs.redomap(cu(lat), op, map="nn_dist", lng=cu(lng), query=q)
+    want = oracle.redomap(lat, op, "nn_dist", lng, q)
+    asum = want if op == "add" else None  # distances are non-negative
+    assert_reduced(got, want, op, asum, "nn")
+    if op == "argmin":
+        assert int(host(got[1])) < workloads.NN_BASE  # first of the 20 copies
+
+
+def test_redomap_nn_misaligned_and_ibase(fs):
+    lat, lng, q = workloads.c2_nn(base=5001, reps=3)
+    got = fs.redomap(cu(lat, 1), "argmin", map="nn_dist", lng=cu(lng, 2), query=q, ibase=1000)
+    v, i = oracle.redomap(lat, "argmin", "nn_dist", lng, q)
+    assert float(host(got[0])) == float(v) and int(host(got[1])) == i + 1000
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("k", [1, 5, 34, 100, 1024, 4096])
+def test_redomap_vadd(fs, dt, k):
+    """VADD(k) over [n][k] = column sums (Fig 4b map(+), G5)."""
+    n = 20_011 if k <= 100 else 3001
+    x = workloads.mixed((n, k), 7 + k, dt)
+    got = fs.redomap(cu(x), "vadd")
+    want = oracle.vreduce(x, "add")
+    asum = oracle.vreduce(np.abs(x), "add") if dt == np.float32 else None
+    assert_reduced(got, want, "add", asum, f"vadd k={k}")
+
+
+def test_redomap_vadd_empty(fs):
+    got = fs.redomap(torch.zeros((0, 7), dtype=torch.float32, device="cuda"), "vadd")
+    assert host(got).tolist() == [0.0] * 7
+
+
+# ------------------------------------------------------------------ combine
+@pytest.mark.parametrize("op", OPS)
+def test_combine(fs, op):
+    parts = workloads.mixed(37, 5, np.float32)
+    parts[3] = parts[30] = parts.min()
+    pidx = np.arange(37, dtype=np.int64) * 1000 + 5
+    got = fs.combine(cu(parts), op, part_idx=cu(pidx) if op == "argmin" else None)
+    want = oracle.reduce(parts, op)
+    if op == "argmin":
+        assert int(host(got[1])) == pidx[want[1]] and float(host(got[0])) == float(want[0])
+    else:
+        assert_reduced(got, want, op, oracle.reduce(np.abs(parts), "add"), "combine")
+
+
+# ------------------------------------------------------------------ scanomap
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("op", OPS)
+@pytest.mark.parametrize("n,offset", [(1, 0), (5, 1), (4096, 0), (100_003, 0), (1_000_003, 2)])
+def test_scanomap(fs, dt, op, n, offset):
+    x = workloads.mixed(n, 200 + n, dt)
+    got = fs.scanomap(cu(x, offset), op)
+    want = oracle.scan(x, op)
+    asum = oracle.scan(np.abs(x), "add") if op == "add" and dt == np.float32 else None
+    assert_reduced(got, want, op, asum, f"scan n={n}")
+
+
+def test_scanomap_full_range_i32_and_carry(fs):
+    x = workloads.c1(1 << 20)
+    np.testing.assert_array_equal(host(fs.scanomap(cu(x), "add")), oracle.scan(x, "add"))
+    # carry-in (F5's accumulator a): scan of the second half continued from the first
+    h = x.size // 2
+    first = fs.scanomap(cu(x[:h]), "add")
+    second = fs.scanomap(cu(x[h:]), "add", carry=first[-1:].clone())
+    np.testing.assert_array_equal(np.concatenate([host(first), host(second)]), oracle.scan(x, "add"))
+    y = workloads.mixed(50_000, 3, np.float32)
+    y[10] = y[40_000] = y.min()
+    a = fs.scanomap(cu(y[:25_000]), "argmin")
+    b = fs.scanomap(cu(y[25_000:]), "argmin", carry=a[0][-1:].clone(), carry_idx=a[1][-1:].clone(), ibase=25_000)
+    wv, wi = oracle.scan(y, "argmin")
+    np.testing.assert_array_equal(np.concatenate([host(a[1]), host(b[1])]), wi)
+    np.testing.assert_array_equal(np.concatenate([host(a[0]), host(b[0])]), wv)
+
+
+@pytest.mark.parametrize("op", ["add", "min", "argmin"])
+def test_scanomap_nn(fs, op):
+    lat, lng, q = workloads.c2_nn(base=30_011, reps=3)
+    got = fs.scanomap(cu(lat), op, map="nn_dist", lng=cu(lng), query=q)
+    want = oracle.scanomap(lat, op, "nn_dist", lng, q)
+    assert_reduced(got, want, op, want if op == "add" else None, "scan nn")
+
+
+# ------------------------------------------------------------------ seg_reduce
+SEG_SHAPES = [(1, 1), (1000, 1), (777, 3), (513, 7), (300, 16), (200, 33), (64, 64), (100, 100), (50, 1000),
+              (9, 4097), (3, 65537), (2, 300_001), (1, 1_000_003)]
+
+
+@pytest.mark.parametrize("nseg,seglen", SEG_SHAPES)
+@pytest.mark.parametrize("regime", [-1, 0, 1, 2, 3])
+def test_seg_reduce_regimes_f32_and_i32(fs, nseg, seglen, regime):
+    fs.force_seg_regime(regime)
+    try:
+        for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "max")):
+            x = workloads.mixed(nseg * seglen, nseg + seglen, dt)
+            got = fs.seg_reduce(cu(x), nseg, seglen, op)
+            want = oracle.seg_reduce(x, nseg, seglen, op)
+            asum = oracle.seg_reduce(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+            assert_reduced(got, want, op, asum, f"seg {nseg}x{seglen} r={regime} {dt.__name__} {op}")
+    finally:
+        fs.force_seg_regime(-1)
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("op", OPS)
+def test_seg_reduce_all_ops_misaligned(fs, dt, op):
+    for nseg, seglen in [(333, 5), (65, 129), (5, 20_001)]:
+        x = workloads.mixed(nseg * seglen, 9, dt)
+        got = fs.seg_reduce(cu(x, 1), nseg, seglen, op)
+        want = oracle.seg_reduce(x, nseg, seglen, op)
+        asum = oracle.seg_reduce(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"seg misaligned {nseg}x{seglen}")
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("op", OPS)
+@pytest.mark.parametrize("nseg,seglen", [(1, 1), (1, 5000), (7, 3), (1000, 50), (5, 20_000), (100_000, 3), (4096, 64)])
+def test_seg_reduce_col_major(fs, dt, op, nseg, seglen):
+    """as_column_major (L1431): same logical rows, stored column-major."""
+    x = workloads.mixed(nseg * seglen, 31, dt)
+    cm = np.ascontiguousarray(x.reshape(nseg, seglen).T).reshape(-1)
+    got = fs.seg_reduce(cu(cm), nseg, seglen, op, layout="col")
+    want = oracle.seg_reduce(cm, nseg, seglen, op, "col")
+    asum = oracle.seg_reduce(np.abs(cm), nseg, seglen, "add", "col") if (op == "add" and dt == np.float32) else None
+    assert_reduced(got, want, op, asum, f"col {nseg}x{seglen}")
+    if dt != np.float32 or op != "add":  # C-13: col(transpose X) == row(X) bit for bit
+        row = fs.seg_reduce(cu(x), nseg, seglen, op)
+        if op == "argmin":
+            np.testing.assert_array_equal(host(row[1]), host(got[1]))
+        else:
+            np.testing.assert_array_equal(host(row), host(got))
+
+
+def test_seg_reduce_empty(fs):
+    for op in OPS:
+        got = fs.seg_reduce(torch.zeros(0, dtype=torch.float32, device="cuda"), 5, 0, op)
+        want = oracle.seg_reduce(np.zeros(0, np.float32), 5, 0, op)
+        if op == "argmin":
+            assert host(got[1]).tolist() == [-1] * 5
+        else:
+            np.testing.assert_array_equal(host(got), want.astype(np.float32))
+    assert fs.seg_reduce(torch.zeros(0, dtype=torch.int32, device="cuda"), 0, 7, "add").numel() == 0
+
+
+# ------------------------------------------------------------------ seg_scan
+@pytest.mark.parametrize("nseg,seglen", [(1, 1), (1000, 1), (777, 3), (300, 16), (200, 33), (50, 1000), (9, 4097),
+                                         (3, 65537), (1, 1_000_003)])
+@pytest.mark.parametrize("layout", ["row", "col"])
+def test_seg_scan(fs, nseg, seglen, layout):
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int32, "max")):
+        x = workloads.mixed(nseg * seglen, nseg * 3 + seglen, dt)
+        got = fs.seg_scan(cu(x), nseg, seglen, op, layout=layout)
+        want = oracle.seg_scan(x, nseg, seglen, op, layout)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", layout) if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan {layout} {nseg}x{seglen} {dt.__name__} {op}")
+
+
+def test_seg_scan_misaligned(fs):
+    x = workloads.mixed(50 * 999, 4, np.int64)
+    got = fs.seg_scan(cu(x, 1), 50, 999, "add")
+    np.testing.assert_array_equal(host(got), oracle.seg_scan(x, 50, 999, "add"))
+
+
+# ------------------------------------------------------------------ stream_red
+@pytest.mark.parametrize("keys", ["uniform", "clustered", "skewed"])
+def test_stream_red_c3_kdd_shape(fs, keys):
+    """BASELINE configs[2]: kdd_cup shape n=494,019, d=34, k=5; counts bit-exact, sums 1e-4."""
+    pts, mem = workloads.c3_kmeans(keys=keys)
+    sums, counts = fs.stream_red(cu(pts), cu(mem), 5)
+    ws, wc = oracle.stream_red(pts, mem, 5)
+    np.testing.assert_array_equal(host(counts), wc)
+    absum, _ = oracle.stream_red(np.abs(pts), mem, 5)
+    assert_reduced(sums, ws, "add", absum, "kmeans c3")
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("k,w", [(1, 1), (3, 7), (8, 32), (5, 33), (16, 64), (32, 34), (32, 64), (33, 10),
+                                 (100, 70), (7, 200), (300, 100), (2000, 40)])
+def test_stream_red_shapes(fs, dt, k, w):
+    n = 30_011
+    vals = workloads.mixed((n, w), k * 100 + w, dt)
+    mem = workloads.ints(n, k + w, 0, k)
+    sums, counts = fs.stream_red(cu(vals), cu(mem), k)
+    ws, wc = oracle.stream_red(vals, mem, k)
+    np.testing.assert_array_equal(host(counts), wc)
+    absum = oracle.stream_red(np.abs(vals), mem, k)[0] if dt == np.float32 else None
+    assert_reduced(sums, ws, "add", absum, f"stream_red k={k} w={w}")
+
+
+def test_stream_red_small_and_empty(fs):
+    for n in (0, 1, 17):
+        vals = workloads.mixed((n, 34), 1, np.float32)
+        mem = workloads.ints(n, 2, 0, 5)
+        sums, counts = fs.stream_red(cu(vals) if n else torch.zeros((0, 34), device="cuda"),
+                                     cu(mem) if n else torch.zeros(0, dtype=torch.int32, device="cuda"), 5)
+        ws, wc = oracle.stream_red(vals, mem, 5)
+        np.testing.assert_array_equal(host(counts), wc)
+        np.testing.assert_allclose(host(sums), ws, rtol=1e-5, atol=1e-6)
+
+
+def test_stream_red_bad_key_raises(fs):
+    vals = workloads.mixed((1000, 4), 1, np.float32)
+    mem = workloads.ints(1000, 2, 0, 5)
+    mem[123] = 9
+    fs.check_device_error()  # clear state
+    fs.stream_red(cu(vals), cu(mem), 5)
+    with pytest.raises(fs.FutsegError, match="BOUNDS"):
+        fs.check_device_error()
+    fs.check_device_error()  # cleared
+
+
+# ------------------------------------------------------------------ transpose
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("r,c", [(1, 1), (1, 1000), (1000, 1), (32, 32), (33, 65), (1000, 777), (4096, 4096)])
+def test_transpose(fs, dt, r, c):
+    x = workloads.mixed((r, c), r + c, dt)
+    got = fs.transpose_2d(cu(x))
+    np.testing.assert_array_equal(host(got), oracle.transpose_2d(x))
+
+
+# ------------------------------------------------------------------ full BASELINE sizes
+_C4 = []
+
+
+def _c4():
+    if not _C4:
+        _C4.append(workloads.c4())
+    return _C4[0]
+
+
+@pytest.mark.slow
+def test_full_c1_seg_reduce_1024x1024(fs):
+    x = workloads.c1()
+    for regime in (-1, 0, 1, 2, 3):
+        fs.force_seg_regime(regime)
+        try:
+            got = fs.seg_reduce(cu(x), 1024, 1024, "add")
+        finally:
+            fs.force_seg_regime(-1)
+        np.testing.assert_array_equal(host(got), oracle.seg_reduce(x, 1024, 1024, "add"))
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("seglen", [1, 32, 1024, 65536, 1 << 28])
+def test_full_c4_seg_reduce_and_scan(fs, seglen):
+    """BASELINE configs[3] at full size (2^28 f32): seg_reduce compared everywhere; seg_scan
+    compared on a sample of 4096 positions plus every segment end."""
+    x = _c4()
+    nseg = (1 << 28) // seglen
+    xt = cu(x)
+    got = host(fs.seg_reduce(xt, nseg, seglen, "add"))
+    want = oracle.seg_reduce(x, nseg, seglen, "add")
+    err = np.abs(got.astype(np.float64) - want)
+    assert np.all(err <= TOL * want + 1e-30), err.max()  # non-negative data: relative bound
+    sc = fs.seg_scan(xt, nseg, seglen, "add")
+    del xt
+    r = workloads.rng(99)
+    pos = np.unique(np.concatenate([r.integers(0, 1 << 28, 4096), np.arange(nseg)[:4096] * seglen + seglen - 1]))
+    gs = host(sc[torch.from_numpy(pos).cuda()]).astype(np.float64)
+    ws = oracle.seg_scan(x, nseg, seglen, "add")[pos] if seglen <= 65536 else oracle.scan(x, "add")[pos]
+    assert np.all(np.abs(gs - ws) <= TOL * ws + 1e-30)
+
+
+@pytest.mark.slow
+def test_full_c5_transpose_and_kmeans(fs):
+    """BASELINE configs[4] single-GPU legs: transpose 2^14 x 2^14 f32 (sampled rows) and the
+    k-means update n=2^26, d=34, k=32 checked against the oracle chunk by chunk (F3 combine)."""
+    from workloads import C5_T
+    x = workloads.device_uniform((C5_T, C5_T), 6, "cuda")
+    t = fs.transpose_2d(x)
+    rows = workloads.rng(5).integers(0, C5_T, 16)
+    for j in rows:
+        np.testing.assert_array_equal(host(t[j]), host(x[:, j]))
+    del x, t
+    pts, mem = workloads.c5_kmeans_shard(0, "cuda")
+    sums, counts = fs.stream_red(pts, mem, 32)
+    ws = np.zeros((32, 34))
+    wc = np.zeros(32, np.int64)
+    chunk = 1 << 22
+    for a in range(0, pts.shape[0], chunk):
+        s, c = oracle.stream_red(host(pts[a:a + chunk]), host(mem[a:a + chunk]), 32)
+        ws += s
+        wc += c
+    np.testing.assert_array_equal(host(counts), wc.astype(np.int32))
+    assert np.all(np.abs(host(sums).astype(np.float64) - ws) <= TOL * ws)
