@@ -1,0 +1,417 @@
+#!/usr/bin/env python
+"""bench.py -- libfutseg hot-path benchmark (one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N
+
+A STEP is one pass of the whole hot path over one
+batch of synthetic input resident in HBM, per GPU (weak scaling: rank r owns
+shard r of an N-times larger global problem, seeds offset by r):
+
+  redomap      f32 add over 2^28 (C4-shaped, 1 GiB)                       A1
+  nn_argmin    Rodinia NN argmin redomap, 855,280 (lat,lng) f32 (C2)      A1
+  scanomap     f32 add inclusive scan over 2^28                            A2
+  stream_red   k-means centre sums+counts, n=2^26, d=34, k=32 (C5)         A3
+  seg_reduce   f32 add, 2^28 elements, seglen 32 / 1024 / 65536 / 2^20
+               (regimes KG1 / KG2 / KG3 / KG4) and column-major seglen 1024 A4
+  seg_scan     f32 add, 2^28 elements, seglen 1024, row-major             A5
+  transpose_2d f32 2^14 x 2^14 (C5)                                        A6
+  combine      at N > 1: all_reduce / all_gather + fs_combine of the
+               partials of redomap, nn_argmin, scanomap carries and
+               stream_red (NCCL over NVLink)                               A7
+
+value = algorithmic bytes of all ranks' steps / max-over-ranks device time
+(GB/s, SURVEY.md 8(d) byte counts).  Every input is larger than L2 except
+the 6.8 MB NN input, which the ~21 GB the rest of the step streams evicts
+between iterations.  See DESIGN.md "Measurement".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GB/s and elements/s per primitive (fraction of B200 HBM peak) at 1/2/4/8 GPUs"
+GB = 1e9
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML while the timed region runs."""
+
+    REASONS = {
+        0x0000000000000001: "gpu_idle", 0x0000000000000002: "applications_clocks_setting",
+        0x0000000000000004: "sw_power_cap", 0x0000000000000008: "hw_slowdown",
+        0x0000000000000020: "sw_thermal_slowdown", 0x0000000000000040: "hw_thermal_slowdown",
+        0x0000000000000080: "hw_power_brake_slowdown", 0x0000000000000100: "display_clocks_setting",
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:  # noqa: BLE001
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                mask = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if mask & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:  # noqa: BLE001
+                pass
+            self._stop.wait(0.05)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ workload
+def build_workload(fs, dev, rank, world, quick):
+    import torch
+    import workloads as wl
+    sh = 4 if quick else 0  # --quick: 16x smaller inputs (for harness checks only)
+    n = (1 << 28) >> sh
+    W = {}
+    W["x"] = wl.device_uniform(n, 5 + 1000 * rank, dev)
+    lat, lng, q = wl.c2_nn(seed=2 + rank)
+    W["lat"], W["lng"], W["q"] = torch.from_numpy(lat).to(dev), torch.from_numpy(lng).to(dev), q
+    W["pts"], W["mem"] = wl.c5_kmeans_shard(rank, dev, n=(1 << 26) >> sh)
+    t = (1 << 14) >> (sh // 2)
+    W["tmat"] = wl.device_uniform((t, t), 6 + 1000 * rank, dev)
+    # preallocated outputs (no allocation inside the timed region)
+    f32 = dict(dtype=torch.float32, device=dev)
+    W["o_red"] = torch.empty((), **f32)
+    W["o_nn"] = (torch.empty((), **f32), torch.empty((), dtype=torch.int64, device=dev))
+    W["o_scan"] = torch.empty(n, **f32)
+    W["o_sums"] = torch.empty((32, 34), **f32)
+    W["o_cnt"] = torch.empty(32, dtype=torch.int32, device=dev)
+    W["o_segscan"] = torch.empty(n, **f32)
+    W["o_tr"] = torch.empty((t, t), **f32)
+    W["seglens"] = [32, 1024, 65536, 1 << 20]
+    W["o_seg"] = {L: torch.empty(n // L, **f32) for L in W["seglens"]}
+    W["o_segcol"] = torch.empty(n // 1024, **f32)
+    W["n"], W["t"] = n, t
+    W["ibase_x"], W["ibase_nn"] = rank * n, rank * lat.size
+    return W
+
+
+def make_step(fs, W, world):
+    """[(name, fn, algorithmic bytes per rank, elements per rank)] for one step."""
+    import torch
+    from paper_conf_pldi_henriksenseho17_b200 import dist as fdist
+    n, t = W["n"], W["t"]
+    nn = W["lat"].numel()
+    kn = W["pts"].shape[0]
+    multi = world > 1
+    st = []
+
+    def red():
+        if multi:
+            fs.redomap(W["x"], "add", out=W["o_red"])
+            torch.distributed.all_reduce(W["o_red"])
+        else:
+            fs.redomap(W["x"], "add", out=W["o_red"])
+
+    def nn_argmin():
+        if multi:
+            fdist.redomap(W["lat"], "argmin", ibase=W["ibase_nn"], map="nn_dist", lng=W["lng"], query=W["q"])
+        else:
+            fs.redomap(W["lat"], "argmin", map="nn_dist", lng=W["lng"], query=W["q"], out=W["o_nn"][0],
+                       out_idx=W["o_nn"][1])
+
+    def scan():
+        if multi:
+            fdist.scanomap(W["x"], "add")  # local total + all_gather + carry-in scan (3n)
+        else:
+            fs.scanomap(W["x"], "add", out=W["o_scan"])
+
+    def kmeans():
+        fs.stream_red(W["pts"], W["mem"], 32, sums=W["o_sums"], counts=W["o_cnt"])
+        if multi:
+            torch.distributed.all_reduce(W["o_sums"])
+            torch.distributed.all_reduce(W["o_cnt"])
+
+    st.append(("redomap_f32_add", red, 4 * n, n))
+    st.append(("nn_argmin_redomap", nn_argmin, 8 * nn, nn))
+    st.append(("scanomap_f32_add", scan, (12 if multi else 8) * n, n))
+    st.append(("stream_red_kmeans_k32_d34", kmeans, (4 * 34 + 4) * kn, kn))
+    for L in W["seglens"]:
+        st.append((f"seg_reduce_row_L{L}",
+                   (lambda L=L: fs.seg_reduce(W["x"], n // L, L, "add", out=W["o_seg"][L])),
+                   4 * n + 4 * (n // L), n))
+    st.append(("seg_reduce_col_L1024", lambda: fs.seg_reduce(W["x"], n // 1024, 1024, "add", layout="col",
+                                                             out=W["o_segcol"]), 4 * n + 4 * (n // 1024), n))
+    st.append(("seg_scan_row_L1024", lambda: fs.seg_scan(W["x"], n // 1024, 1024, "add", out=W["o_segscan"]),
+               8 * n, n))
+    st.append(("transpose_2d_f32", lambda: fs.transpose_2d(W["tmat"], out=W["o_tr"]), 8 * t * t, t * t))
+    return st
+
+
+# ------------------------------------------------------------------ cpu baseline (oracle)
+def oracle_sample(W, scale_shift):
+    """Host copies of a bounded sample of every primitive's input (same data as the GPU run)."""
+    s = {}
+    m = min(W["n"], (1 << 25) >> scale_shift)
+    s["x"] = W["x"][:m].cpu().numpy()
+    s["lat"], s["lng"] = W["lat"].cpu().numpy(), W["lng"].cpu().numpy()
+    kr = min(W["pts"].shape[0], (1 << 21) >> scale_shift)
+    s["pts"], s["mem"] = W["pts"][:kr].cpu().numpy(), W["mem"][:kr].cpu().numpy()
+    tt = min(W["t"], 4096 >> (scale_shift // 2))
+    s["tmat"] = W["tmat"][:tt, :tt].cpu().numpy()
+    return s
+
+
+def oracle_step(s, q):
+    """One pass of the oracle over the sample; returns (algorithmic bytes, seconds)."""
+    import oracle
+    x = s["x"]
+    m = x.size
+    t0 = time.perf_counter()
+    oracle.reduce(x, "add")
+    oracle.redomap(s["lat"], "argmin", "nn_dist", s["lng"], q)
+    oracle.scan(x, "add")
+    oracle.stream_red(s["pts"], s["mem"], 32)
+    for L in (32, 1024, 65536):
+        oracle.seg_reduce(x, m // L, L, "add")
+    oracle.seg_reduce(x, m // 1024, 1024, "add", "col")
+    oracle.seg_scan(x, m // 1024, 1024, "add")
+    oracle.transpose_2d(s["tmat"])
+    dt = time.perf_counter() - t0
+    kr = s["mem"].size
+    tt = s["tmat"].shape[0]
+    nbytes = (4 * m + 8 * s["lat"].size + 8 * m + 140 * kr + 3 * (4 * m) + sum(4 * (m // L) for L in (32, 1024, 65536))
+              + 4 * m + 4 * (m // 1024) + 8 * m + 8 * tt * tt)
+    return nbytes, dt, f"{m} f32 (redomap, scan, seg ops L=32/1024/65536/col, seg_scan), NN {s['lat'].size} " \
+                       f"records, k-means {kr}x34 k=32, transpose {tt}x{tt}"
+
+
+def run_reference(args):
+    """--impl reference: the oracle (the only reference this tier has), timed on host cores."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import torch
+    import workloads as wl
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    W = {"x": wl.device_uniform(1 << 23, 5, dev), "lat": None}
+    lat, lng, q = wl.c2_nn(seed=2)
+    W["lat"], W["lng"] = torch.from_numpy(lat), torch.from_numpy(lng)
+    W["pts"], W["mem"] = wl.c5_kmeans_shard(0, dev, n=1 << 19)
+    W["tmat"] = wl.device_uniform((2048, 2048), 6, dev)
+    W["n"], W["t"] = 1 << 23, 2048
+    s = oracle_sample(W, 0)
+    for _ in range(args.warmup):
+        oracle_step(s, q)
+    tot_b, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        b, dt, desc = oracle_step(s, q)
+        tot_b += b
+        tot_t += dt
+    val = tot_b / tot_t / GB
+    line = {"impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * tot_t / args.steps, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64-accumulated (f32 in)",
+            "data": "synthetic",
+            "config": {"workload": "libfutseg hot-path suite (bounded oracle sample per step)", "sample": desc},
+            "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+            "e2e": {"value": round(val, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--quick", action="store_true", help="16x smaller inputs (harness check; not a bench value)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--only", default="", help="comma-separated primitive names (profiling aid)")
+    args = ap.parse_args()
+    if args.warmup < 3 and not args.quick and not args.only:
+        print("bench.py: --warmup must be >= 3", file=sys.stderr)
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as tdist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch N>1 with torch.distributed.run",
+              file=sys.stderr)
+        sys.exit(2)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        tdist.init_process_group("nccl", device_id=dev)
+    import paper_conf_pldi_henriksenseho17_b200 as fs
+
+    W = build_workload(fs, dev, rank, world, args.quick)
+    steps = make_step(fs, W, world)
+    if args.only:
+        keep = set(args.only.split(","))
+        steps = [s for s in steps if s[0] in keep]
+    names = [s[0] for s in steps]
+
+    def barrier():
+        if world > 1:
+            tdist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        for _, fn, _, _ in steps:
+            fn()
+    barrier()
+
+    K = args.steps
+    ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in steps]
+          for _ in range(K)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = fs.launch_count()
+    with ClockSampler(local) as clk:
+        barrier()
+        start.record()
+        for s in range(K):
+            for p, (_, fn, _, _) in enumerate(steps):
+                ev[s][p][0].record()
+                fn()
+                ev[s][p][1].record()
+        end.record()
+        barrier()
+    launches = fs.launch_count() - l0
+    total_ms = start.elapsed_time(end)
+    tmax = torch.tensor([total_ms], device=dev, dtype=torch.float64)
+    if world > 1:
+        tdist.all_reduce(tmax, op=tdist.ReduceOp.MAX)
+    total_ms = float(tmax.item())
+    per = {}
+    for p, (name, _, nbytes, nel) in enumerate(steps):
+        ms = [ev[s][p][0].elapsed_time(ev[s][p][1]) for s in range(K)]
+        avg = sum(ms) / K
+        per[name] = {"ms": round(avg, 4), "ms_min": round(min(ms), 4), "GB_s": round(nbytes / (avg * 1e-3) / GB, 1),
+                     "elements_per_s": float(f"{nel / (avg * 1e-3):.4g}"), "bytes": nbytes}
+    step_bytes = sum(s[2] for s in steps)
+    step_elems = sum(s[3] for s in steps)
+    value = step_bytes * world * K / (total_ms * 1e-3) / GB
+    peak, peak_src = peaks()
+    for name in per:
+        per[name]["frac_of_peak"] = round(per[name]["GB_s"] / peak, 4)
+    dom = max(per, key=lambda k: per[k]["ms"])
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tf):
+        with open(tf) as f:
+            traffic = json.load(f).get(dom)
+
+    # ---------------- e2e: host buffers, H2D + compute + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e and not args.only:
+        host_in = {k: W[k].cpu().pin_memory() for k in ("x", "lat", "lng", "pts", "mem", "tmat")}
+        outs = [W["o_red"], W["o_nn"][0], W["o_nn"][1], W["o_scan"], W["o_sums"], W["o_cnt"], W["o_segscan"],
+                W["o_tr"], W["o_segcol"]] + list(W["o_seg"].values())
+        host_out = [torch.empty(o.shape, dtype=o.dtype, pin_memory=True) for o in outs]
+        h2d = sum(v.numel() * v.element_size() for v in host_in.values())
+        d2h = sum(o.numel() * o.element_size() for o in outs)
+        KE = max(1, args.e2e_steps)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(KE):
+            for k, v in host_in.items():
+                W[k].copy_(v, non_blocking=True)
+            for _, fn, _, _ in steps:
+                fn()
+            for o, h in zip(outs, host_out):
+                h.copy_(o, non_blocking=True)
+        e1.record()
+        barrier()
+        ems = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
+        if world > 1:
+            tdist.all_reduce(ems, op=tdist.ReduceOp.MAX)
+        e2e = {"value": round(step_bytes * world * KE / (float(ems.item()) * 1e-3) / GB, 2), "unit": "GB/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": KE,
+               "note": "same algorithmic bytes; pinned host inputs copied in and all outputs copied out every step"}
+
+    # ---------------- cpu baseline: the oracle on a bounded sample, rank 0, N = 1
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.only:
+        s = oracle_sample(W, 4 if args.quick else 0)
+        b, dt, desc = oracle_step(s, W["q"])
+        cpu = {"value": round(b / dt / GB, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": desc, "seconds": round(dt, 2)}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": round(total_ms / K, 4), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "libfutseg hot-path suite: redomap 2^28 f32, NN argmin 855,280 (C2), scanomap 2^28, "
+                                   "k-means stream_red 2^26x34 k=32 (C5), seg_reduce 2^28 L=32/1024/65536/2^20 row + "
+                                   "L=1024 col, seg_scan 2^28 L=1024, transpose 2^14^2 f32 (C5)" +
+                                   (" [QUICK 1/16 sizes]" if args.quick else ""),
+                       "per_rank_bytes_per_step": step_bytes, "per_rank_elements_per_step": step_elems,
+                       "l2": "inputs > L2 (126 MB) except NN (6.8 MB), evicted by the ~21 GB rest of each step",
+                       "parallelism": f"dp{world} (weak: one shard per GPU)", "elements_per_s":
+                           float(f"{step_elems * world * K / (total_ms * 1e-3):.4g}")},
+            "roofline": {"bound": "hbm", "kernel": dom, "achieved": per[dom]["GB_s"], "peak": peak, "unit": "GB/s",
+                         "frac": round(per[dom]["GB_s"] / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                         "bytes_per_launch": per[dom]["bytes"]},
+            "per_primitive": per,
+            "clocks": clk.summary(),
+            "gpu_launches": launches,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -221,6 +221,10 @@ fs_status fs_force_seg_regime(int32_t regime);
 const char *fs_status_string(fs_status s);
 const char *fs_version(void);
 
+/* Number of kernels this library has launched in this process (all devices,
+ * all streams).  A benchmark reads it around its timed region. */
+uint64_t fs_launch_count(void);
+
 #ifdef __cplusplus
 }
 #endif

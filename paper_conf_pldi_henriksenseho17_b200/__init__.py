@@ -33,7 +33,7 @@ _LIB_PATH = os.path.join(_HERE, "libfutseg.so")
 if not os.path.exists(_LIB_PATH):
     raise ImportError(
         f"libfutseg.so not found at {_LIB_PATH}; build it with "
-        "`python -m paper_conf_pldi_henriksenseho17_b200.build` (or __graft_entry__.build())")
+        "`python paper_conf_pldi_henriksenseho17_b200/build.py` (or __graft_entry__.build())")
 
 _lib = ctypes.CDLL(_LIB_PATH)
 
@@ -73,6 +73,7 @@ _SIG = {
     "fs_force_seg_regime": [_I],
     "fs_status_string": [_I],
     "fs_version": [],
+    "fs_launch_count": [],
 }
 for _name, _args in _SIG.items():
     _f = getattr(_lib, _name)
@@ -80,6 +81,7 @@ for _name, _args in _SIG.items():
     _f.restype = _I
 _lib.fs_status_string.restype = ctypes.c_char_p
 _lib.fs_version.restype = ctypes.c_char_p
+_lib.fs_launch_count.restype = ctypes.c_uint64
 
 C = _lib  # raw C ABI (ctypes), for callers that manage their own device pointers
 
@@ -101,6 +103,11 @@ def library_path() -> str:
 
 def version() -> str:
     return _lib.fs_version().decode()
+
+
+def launch_count() -> int:
+    """Kernels launched by libfutseg in this process so far."""
+    return int(_lib.fs_launch_count())
 
 
 # ------------------------------------------------------------------ helpers

@@ -1,6 +1,6 @@
 """Build libfutseg.so in-tree (sm_100a) with nvcc.
 
-    python -m paper_conf_pldi_henriksenseho17_b200.build [--force] [-v]
+    python paper_conf_pldi_henriksenseho17_b200/build.py [--force] [-v]
 
 Every csrc/*.cu is compiled separately (in parallel) with
 ``-gencode arch=compute_100a,code=sm_100a -O3 -lineinfo`` and linked into

@@ -4,6 +4,7 @@
 // status has no side effects (mirrors Futhark's hoisted dynamic shape and
 // bounds checks, L429-432).  The launchers it calls live in the per-kernel
 // translation units.
+#include <atomic>
 #include <mutex>
 #include <stdlib.h>
 #include <unordered_map>
@@ -43,6 +44,9 @@ int max_blocks_per_sm(const void *kernel, int threads, size_t smem) {
     cache[key] = b;
     return b;
 }
+
+static std::atomic<unsigned long long> g_launches{0};
+void note_launches(int n) { g_launches.fetch_add((unsigned long long)n, std::memory_order_relaxed); }
 
 static int g_forced_regime = -2;
 int forced_seg_regime() {
@@ -128,6 +132,8 @@ int64_t in_bytes(const fs_opdesc &op, const fs_mapdesc &map, int64_t n) {
 extern "C" {
 
 const char *fs_version(void) { return "libfutseg 0.1 (sm_100a)"; }
+
+uint64_t fs_launch_count(void) { return (uint64_t)g_launches.load(std::memory_order_relaxed); }
 
 const char *fs_status_string(fs_status s) {
     switch (s) {

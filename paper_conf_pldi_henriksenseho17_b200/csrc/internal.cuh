@@ -18,7 +18,9 @@ inline int resident_blocks(const void *kernel, int threads, size_t smem = 0) {
 }
 int forced_seg_regime();  // -1 = automatic
 
-inline fs_status launch_status() {
+void note_launches(int n);  // counts kernels launched by this library (fs_launch_count)
+inline fs_status launch_status(int kernels = 1) {
+    note_launches(kernels);
     return cudaGetLastError() == cudaSuccess ? FS_OK : FS_ERR_CUDA;
 }
 

@@ -470,7 +470,7 @@ template <int OP, typename T> struct ColScanRun {
         colscan_carry_kernel<OP, T><<<(unsigned)g2, 128, 0, st>>>(parts, w, p.Y);
         colscan_kernel<OP, T, VEC, true><<<grid, kColScanThreads, 0, st>>>(x, m, w, p.WV, p.Y, p.rpu, parts, out,
                                                                            out_idx);
-        return launch_status();
+        return launch_status(3);
     }
     static fs_status run(const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx, void *ws, cudaStream_t st) {
         const bool aligned = ((uintptr_t)in & 15) == 0 && ((uintptr_t)out & 15) == 0;

@@ -20,8 +20,8 @@ HEADER = os.path.join(ROOT, "include", "futseg.h")
 
 @pytest.fixture(scope="module")
 def fs():
-    from paper_conf_pldi_henriksenseho17_b200 import build
-    build.build()
+    import __graft_entry__
+    __graft_entry__.build()
     import paper_conf_pldi_henriksenseho17_b200 as m
     return m
 
