@@ -28,7 +28,8 @@
 namespace fs {
 
 // ---------------------------------------------------------------- segmented value
-template <class O> struct SOp {
+// S = (value, flag).  Without SEG the flag is the constant 0 and vanishes.
+template <class O, bool SEG> struct SOp {
     using V = typename O::V;
     struct S {
         V v;
@@ -36,27 +37,20 @@ template <class O> struct SOp {
     };
     static __device__ __forceinline__ S id() { return S{O::id(), 0}; }
     // ordered: a is the left operand
-    static __device__ __forceinline__ S comb(S a, S b) { return b.f ? b : S{O::comb(a.v, b.v), a.f}; }
+    static __device__ __forceinline__ S comb(S a, S b) {
+        if constexpr (SEG) return b.f ? b : S{O::comb(a.v, b.v), a.f};
+        else return S{O::comb(a.v, b.v), 0};
+    }
+    static __device__ __forceinline__ S up(S a, int d) {
+        return S{shfl_up(a.v, d), SEG ? __shfl_up_sync(0xffffffffu, a.f, d) : 0};
+    }
+    static __device__ __forceinline__ S down(S a, int d) {
+        return S{shfl_down_v(a.v, d), SEG ? __shfl_down_sync(0xffffffffu, a.f, d) : 0};
+    }
+    static __device__ __forceinline__ S bcast(S a, int l) {
+        return S{shfl_idx(a.v, l), SEG ? __shfl_sync(0xffffffffu, a.f, l) : 0};
+    }
 };
-
-template <class S> __device__ __forceinline__ S shfl_up_s(S a, int d) {
-    S r;
-    r.v = shfl_up(a.v, d);
-    r.f = __shfl_up_sync(0xffffffffu, a.f, d);
-    return r;
-}
-template <class S> __device__ __forceinline__ S shfl_down_s(S a, int d) {
-    S r;
-    r.v = shfl_down_v(a.v, d);
-    r.f = __shfl_down_sync(0xffffffffu, a.f, d);
-    return r;
-}
-template <class S> __device__ __forceinline__ S shfl_idx_s(S a, int l) {
-    S r;
-    r.v = shfl_idx(a.v, l);
-    r.f = __shfl_sync(0xffffffffu, a.f, l);
-    return r;
-}
 
 __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     unsigned v;
@@ -66,6 +60,19 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
 __device__ __forceinline__ void st_release(unsigned *p, unsigned v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+__device__ __forceinline__ uint64_t ld_relaxed64(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed64(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t to_bits(int32_t v) { return (uint32_t)v; }
+__device__ __forceinline__ uint32_t to_bits(float v) { return __float_as_uint(v); }
+template <typename V> __device__ __forceinline__ V from_bits(uint32_t b);
+template <> __device__ __forceinline__ int32_t from_bits<int32_t>(uint32_t b) { return (int32_t)b; }
+template <> __device__ __forceinline__ float from_bits<float>(uint32_t b) { return __uint_as_float(b); }
 
 template <class S> __device__ __forceinline__ void st_payload(S *p, S a) {
     st_cg(&p->v, a.v);
@@ -78,75 +85,133 @@ template <class S> __device__ __forceinline__ S ld_payload(const S *p) {
     return a;
 }
 
+// Published per-tile state of the decoupled look-back.  Status: 0 = nothing,
+// 1 = tile aggregate, 2 = inclusive prefix.
+//  PACK (4-byte accumulators): one 64-bit word = value bits << 32 | flag << 2 |
+//        status, written and read with single relaxed 64-bit accesses (the
+//        value travels with its status: one L2 round trip per look-back step).
+//  otherwise: a status word released after the payload is stored.
+template <class S, bool PACK> struct TileState;
+template <class S> struct TileState<S, true> {
+    uint64_t *w;
+    __device__ __forceinline__ void publish(int64_t t, S s, unsigned st) const {
+        st_relaxed64(w + t, ((uint64_t)to_bits(s.v) << 32) | (s.f ? 4ull : 0ull) | st);
+    }
+    __device__ __forceinline__ unsigned poll(int64_t t, S &s) const {
+        const uint64_t x = ld_relaxed64(w + t);
+        s.v = from_bits<decltype(s.v)>((uint32_t)(x >> 32));
+        s.f = (int)((x >> 2) & 1);
+        return (unsigned)(x & 3);
+    }
+};
+template <class S> struct TileState<S, false> {
+    uint64_t *w;  // status words (u32) at w, then aggs S[ntiles], incls S[ntiles]
+    S *aggs, *incls;
+    __device__ __forceinline__ void publish(int64_t t, S s, unsigned st) const {
+        st_payload((st == 1 ? aggs : incls) + t, s);
+        st_release((unsigned *)w + t, st);
+    }
+    __device__ __forceinline__ unsigned poll(int64_t t, S &s) const {
+        const unsigned st = ld_acquire((const unsigned *)w + t);
+        if (st == 1) s = ld_payload(aggs + t);
+        else if (st == 2) s = ld_payload(incls + t);
+        return st;
+    }
+};
+
 __device__ __forceinline__ float nn_dist_s(float lat, float lng, float q0, float q1) {
     const float d0 = __fsub_rn(lat, q0), d1 = __fsub_rn(lng, q1);
     return __fsqrt_rn(__fadd_rn(__fmul_rn(d0, d0), __fmul_rn(d1, d1)));
 }
 
 constexpr int kScanThreads = 256;
-constexpr int kScanRows = 4;  // 16-byte vectors per lane per tile
 constexpr unsigned kStAgg = 1, kStIncl = 2;
 
-// ws body layout (after the 256-byte header):
-//   [0, 256)                 : tile counter
-//   [256, 256 + st_bytes)    : status words (u32 per tile)
-//   then aggregates S[ntiles], inclusive prefixes S[ntiles]
-struct ScanWs {
-    unsigned *counter, *status;
-    void *aggs, *incls;
-    size_t clear_bytes;
+// 16-byte vectors per lane per tile: 8 for 8-byte (value, flag) pairs, 4 for wider ones
+template <int OP, typename T> struct ScanShape {
+    static constexpr bool PACK = OP != kArgmin && sizeof(T) == 4;
+    static constexpr int R = (OP != kArgmin && sizeof(T) == 4) ? 8 : 4;
+    static constexpr int VEC = 16 / sizeof(T);
+    static constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
+    static constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
 };
-template <class S> static ScanWs scan_ws_layout(void *ws, int64_t ntiles) {
-    char *b = (char *)ws + kWsHeader;
-    ScanWs w;
-    w.counter = (unsigned *)b;
-    w.status = (unsigned *)(b + 256);
-    const size_t st = align_up((size_t)ntiles * 4, 256);
-    w.aggs = b + 256 + st;
-    w.incls = b + 256 + st + align_up((size_t)ntiles * sizeof(S), 256);
-    w.clear_bytes = 256 + st;
-    return w;
-}
 
-template <int OP, typename T, bool NN, bool SEG, bool ALIGNED>
-__global__ void __launch_bounds__(kScanThreads)
-scan_lookback_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n, int64_t L, float q0,
-                     float q1, int64_t ibase, T *__restrict__ out, int64_t *__restrict__ out_idx, const T *carry,
-                     const int64_t *carry_idx, unsigned *counter, unsigned *status,
-                     typename SOp<Op<OP, T>>::S *aggs, typename SOp<Op<OP, T>>::S *incls, int64_t ntiles) {
+// One pass: every CTA repeatedly takes the next tile id (atomic counter, so all
+// predecessors are owned by running CTAs), prefetches the FOLLOWING tile with a
+// TMA bulk copy into its second shared-memory buffer, scans the current tile,
+// runs the decoupled look-back (warp 0) and writes the tile.  With TMA the next
+// tile's HBM read overlaps this tile's scan, look-back and store.
+template <int OP, typename T, bool NN, bool SEG, bool TMA>
+__global__ void __launch_bounds__(kScanThreads, TMA ? 3 : 2)
+scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n, int64_t L, float q0, float q1,
+            int64_t ibase, T *__restrict__ out, int64_t *__restrict__ out_idx, const T *carry,
+            const int64_t *carry_idx, unsigned *counter, TileState<typename SOp<Op<OP, T>, SEG>::S,
+                                                                   ScanShape<OP, T>::PACK> ts,
+            int64_t ntiles, bool aligned) {
     using O = Op<OP, T>;
-    using SO = SOp<O>;
+    using SO = SOp<O, SEG>;
     using S = typename SO::S;
-    constexpr int VEC = 16 / sizeof(T);
-    constexpr int R = kScanRows;
-    constexpr int NW = kScanThreads / 32;
-    constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
-    __shared__ S s_wtot[NW];
-    __shared__ S s_wex[NW];
-    __shared__ S s_ex;
-    __shared__ int64_t s_tile;
+    using Sh = ScanShape<OP, T>;
+    constexpr int VEC = Sh::VEC, R = Sh::R, NW = kScanThreads / 32;
+    constexpr int64_t TILE = Sh::TILE;
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    __shared__ uint64_t bars[2];
+    __shared__ int64_t s_tile[2];
+    __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_val[NW];
+    __shared__ int s_lb_min[NW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
 
-    while (true) {
-        if (threadIdx.x == 0) s_tile = (int64_t)atomicAdd(counter, 1u);
-        __syncthreads();
-        const int64_t tile = s_tile;
+    if (threadIdx.x == 0) {
+        if (TMA) {
+            mbar_init(&bars[0], 1);
+            mbar_init(&bars[1], 1);
+            fence_mbar_init();
+        }
+        const int64_t t0 = (int64_t)atomicAdd(counter, 1u);
+        s_tile[0] = t0;
+        if (TMA && t0 < ntiles && (t0 + 1) * TILE <= n) {
+            mbar_expect_tx(&bars[0], Sh::TILE_BYTES);
+            tma_load_1d(sbuf, in0 + t0 * TILE, Sh::TILE_BYTES, &bars[0]);
+        }
+    }
+    __syncthreads();
+    for (int it = 0;; ++it) {
+        const int b = it & 1;
+        const int64_t tile = s_tile[b];
         if (tile >= ntiles) break;
+        if (threadIdx.x == 0) {
+            const int64_t t1 = (int64_t)atomicAdd(counter, 1u);
+            s_tile[b ^ 1] = t1;
+            if (TMA && t1 < ntiles && (t1 + 1) * TILE <= n) {
+                fence_proxy_async();
+                mbar_expect_tx(&bars[b ^ 1], Sh::TILE_BYTES);
+                tma_load_1d(sbuf + (b ^ 1) * Sh::TILE_BYTES, in0 + t1 * TILE, Sh::TILE_BYTES, &bars[b ^ 1]);
+            }
+        }
+        const bool full = (tile + 1) * TILE <= n;
+        if (TMA && full) mbar_wait(&bars[b], (unsigned)(it >> 1) & 1u);
         const int64_t wbase = tile * TILE + (int64_t)warp * 32 * R * VEC;
 
-        S loc[R][VEC];
+        // phase A: lane totals per row (the tile stays in shared memory with TMA,
+        // otherwise its (mapped) values stay in registers), ordered warp scans
+        T xs[TMA ? 1 : R][VEC];
         S pre[R];
         S carry_w = SO::id();
 #pragma unroll
         for (int q = 0; q < R; ++q) {
             const int64_t p0 = wbase + ((int64_t)q * 32 + lane) * VEC;
             T x[VEC];
-            if (ALIGNED && p0 + VEC <= n) {
+            if (TMA && full) {
+                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(
+                    sbuf + b * Sh::TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+            } else if (aligned && p0 + VEC <= n) {
                 if (NN) {
                     const Vec16<float> a = as_vec<float>(ldg16((const float *)in0 + p0));
-                    const Vec16<float> b = as_vec<float>(ldg16(in1 + p0));
+                    const Vec16<float> c = as_vec<float>(ldg16(in1 + p0));
 #pragma unroll
-                    for (int k = 0; k < VEC; ++k) x[k] = (T)nn_dist_s(a.e[k], b.e[k], q0, q1);
+                    for (int k = 0; k < VEC; ++k) x[k] = (T)nn_dist_s(a.e[k], c.e[k], q0, q1);
                 } else {
                     const Vec16<T> a = as_vec<T>(ldg16(in0 + p0));
 #pragma unroll
@@ -162,6 +227,10 @@ scan_lookback_kernel(const T *__restrict__ in0, const float *__restrict__ in1, i
                         x[k] = T(0);
                     }
                 }
+            }
+            if (!TMA) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) xs[TMA ? 0 : q][k] = x[k];
             }
             int64_t r = SEG ? (p0 % L) : 0;
             S run = SO::id();
@@ -179,93 +248,122 @@ scan_lookback_kernel(const T *__restrict__ in0, const float *__restrict__ in1, i
                     if (r == L) r = 0;
                 }
                 run = SO::comb(run, e);
-                loc[q][k] = run;
             }
             // ordered inclusive warp scan of the lane totals
             S a = run;
 #pragma unroll
             for (int off = 1; off < 32; off <<= 1) {
-                const S o = shfl_up_s(a, off);
+                const S o = SO::up(a, off);
                 if (lane >= off) a = SO::comb(o, a);
             }
-            S ex = shfl_up_s(a, 1);
+            S ex = SO::up(a, 1);
             if (lane == 0) ex = SO::id();
             pre[q] = SO::comb(carry_w, ex);
-            carry_w = SO::comb(carry_w, shfl_idx_s(a, 31));
+            carry_w = SO::comb(carry_w, SO::bcast(a, 31));
         }
         if (lane == 0) s_wtot[warp] = carry_w;
         __syncthreads();
-        if (warp == 0) {
+        // block aggregate and per-warp exclusive prefixes (every warp computes them)
+        S agg;
+        {
             S a = lane < NW ? s_wtot[lane] : SO::id();
 #pragma unroll
             for (int off = 1; off < 32; off <<= 1) {
-                const S o = shfl_up_s(a, off);
+                const S o = SO::up(a, off);
                 if (lane >= off) a = SO::comb(o, a);
             }
-            S wex = shfl_up_s(a, 1);
+            S wex = SO::up(a, 1);
             if (lane == 0) wex = SO::id();
-            if (lane < NW) s_wex[lane] = wex;
-            const S agg = shfl_idx_s(a, NW - 1);
-            // ---- decoupled look-back
-            S exc = SO::id();
-            if (tile == 0) {
-                if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-                if (lane == 0) {
-                    st_payload(incls, SO::comb(exc, agg));
-                    __threadfence();
-                    st_release(status, kStIncl);
-                }
-            } else {
-                if (lane == 0) {
-                    st_payload(aggs + tile, agg);
-                    __threadfence();
-                    st_release(status + tile, kStAgg);
-                }
-                int64_t j = tile - 1;
-                while (true) {
-                    const int64_t idx = j - lane;
-                    unsigned st = kStIncl;
-                    if (idx >= 0) {
-                        st = ld_acquire(status + idx);
-                        while (st == 0) st = ld_acquire(status + idx);
-                    }
-                    const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
-                    const int kk = m ? __ffs(m) - 1 : 31;
-                    S v = SO::id();
-                    if (lane <= kk && idx >= 0) v = (st == kStIncl) ? ld_payload(incls + idx) : ld_payload(aggs + idx);
-                    // ordered reduction: higher lanes are further left
-#pragma unroll
-                    for (int off = 1; off < 32; off <<= 1) {
-                        const S o = shfl_down_s(v, off);
-                        if (lane + off < 32) v = SO::comb(o, v);
-                    }
-                    exc = SO::comb(shfl_idx_s(v, 0), exc);
-                    if (m || exc.f) break;
-                    j -= 32;
-                }
-                if (lane == 0) {
-                    st_payload(incls + tile, SO::comb(exc, agg));
-                    __threadfence();
-                    st_release(status + tile, kStIncl);
-                }
-            }
-            if (lane == 0) s_ex = exc;
+            if (warp == 0 && lane < NW) s_wex[lane] = wex;
+            agg = SO::bcast(a, NW - 1);
         }
+        // ---- decoupled look-back with the whole CTA: 256 predecessors per step
+        // (all CTAs start together, so the nearest published inclusive prefix is
+        // about one wave of resident tiles back; one step covers most of it)
+        S exc = SO::id();
+        if (tile == 0) {
+            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+            if (threadIdx.x == 0) ts.publish(0, SO::comb(exc, agg), kStIncl);
+        } else {
+            if (threadIdx.x == 0) ts.publish(tile, agg, kStAgg);
+            int64_t j = tile - 1;
+            while (true) {
+                const int64_t idx = j - threadIdx.x;
+                S v = SO::id();
+                unsigned st = kStIncl;
+                if (idx >= 0) {
+                    do {
+                        st = ts.poll(idx, v);
+                    } while (st == 0);
+                }
+                // nearest predecessor holding an inclusive prefix
+                const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
+                if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
+                __syncthreads();
+                int kk = 1 << 20;
+#pragma unroll
+                for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
+                if ((int)threadIdx.x > kk || idx < 0) v = SO::id();
+                // ordered reduction: higher thread ids are further left
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const S o = SO::down(v, off);
+                    if (lane + off < 32) v = SO::comb(o, v);
+                }
+                if (lane == 0) s_lb_val[warp] = v;
+                __syncthreads();
+                S P = SO::id();
+#pragma unroll
+                for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_val[q]);
+                exc = SO::comb(P, exc);
+                __syncthreads();  // s_lb_* reuse
+                if (kk < (1 << 20) || exc.f) break;
+                j -= kScanThreads;
+            }
+            if (threadIdx.x == 0) ts.publish(tile, SO::comb(exc, agg), kStIncl);
+        }
+        if (threadIdx.x == 0) s_ex = exc;
         __syncthreads();
+        // phase C: re-derive every element's inclusive value from the tile prefix
         const S base = SO::comb(s_ex, s_wex[warp]);
 #pragma unroll
         for (int q = 0; q < R; ++q) {
             const int64_t p0 = wbase + ((int64_t)q * 32 + lane) * VEC;
-            const S P = SO::comb(base, pre[q]);
+            T x[VEC];
+            if (TMA && full) {
+                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(
+                    sbuf + b * Sh::TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+            } else if (TMA) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in0[p0 + k] : T(0);
+            } else {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) x[k] = xs[TMA ? 0 : q][k];
+            }
+            S run = SO::comb(base, pre[q]);
+            int64_t r = SEG ? (p0 % L) : 0;
             T y[VEC];
             int64_t yi[VEC];
 #pragma unroll
             for (int k = 0; k < VEC; ++k) {
-                const S o = SO::comb(P, loc[q][k]);
-                y[k] = O::val(o.v);
-                yi[k] = O::idx(o.v);
+                S e;
+                if (p0 + k < n) {
+                    e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
+                    e.f = SEG ? (r == 0) : 0;
+                } else {
+                    e = SO::id();
+                }
+                if (SEG) {
+                    ++r;
+                    if (r == L) r = 0;
+                }
+                run = SO::comb(run, e);
+                y[k] = O::val(run.v);
+                yi[k] = O::idx(run.v);
             }
-            if (ALIGNED && p0 + VEC <= n) {
+            if (aligned && p0 + VEC <= n) {
                 Vec16<T> w;
 #pragma unroll
                 for (int k = 0; k < VEC; ++k) w.e[k] = y[k];
@@ -283,25 +381,283 @@ scan_lookback_kernel(const T *__restrict__ in0, const float *__restrict__ in1, i
                     if (p0 + k < n) out_idx[p0 + k] = yi[k];
             }
         }
-        __syncthreads();  // s_tile / smem reuse
+        __syncthreads();  // smem buffers, s_tile and s_ex reuse
     }
 }
 
+// ---------------------------------------------------------------- pipelined TMA scan
+// Software pipeline over the CTA's tiles T0, T1, ... (ids from the atomic
+// counter).  Iteration k:
+//   1. take T(k+1) and start its TMA bulk load into the other buffer
+//   2. look-back for T(k) (its aggregate was published one step earlier)
+//   3. wait for T(k+1); local scan; publish T(k+1)'s aggregate
+//   4. write T(k) = its exclusive prefix (+) local scan (re-derived from smem)
+// A tile's aggregate is published about one look-back after the tile was
+// taken, so successors rarely spin, and the HBM read of T(k+1) overlaps the
+// look-back and output of T(k).
+template <int OP, typename T, bool SEG>
+__global__ void __launch_bounds__(kScanThreads, 3)
+scan_pipe_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+                 int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
+                 TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
+    using O = Op<OP, T>;
+    using SO = SOp<O, SEG>;
+    using S = typename SO::S;
+    using Sh = ScanShape<OP, T>;
+    constexpr int VEC = Sh::VEC, R = Sh::R, NW = kScanThreads / 32;
+    constexpr int64_t TILE = Sh::TILE;
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    __shared__ uint64_t bars[2];
+    __shared__ int64_t s_tile[2];
+    __shared__ S s_wtot[NW], s_wex[2][NW], s_agg[2], s_ex, s_lb_val[NW];
+    __shared__ int s_lb_min[NW];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+
+    // element k of this lane's vector in row q of tile `tile` (buffer b)
+    auto load_row = [&](int b, int64_t tile, int q, T (&x)[VEC]) {
+        const int64_t p0 = tile * TILE + (int64_t)warp * 32 * R * VEC + ((int64_t)q * 32 + lane) * VEC;
+        if ((tile + 1) * TILE <= n) {
+            const Vec16<T> a =
+                *reinterpret_cast<const Vec16<T> *>(sbuf + b * Sh::TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+        } else {
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
+        }
+        return p0;
+    };
+    auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
+        S e;
+        if (p0 + k < n) {
+            e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
+            e.f = SEG ? (r == 0) : 0;
+        } else {
+            e = SO::id();
+        }
+        if (SEG) {
+            ++r;
+            if (r == L) r = 0;
+        }
+        return e;
+    };
+    auto issue = [&](int b, int64_t tile) {  // thread 0
+        if (tile < ntiles && (tile + 1) * TILE <= n) {
+            fence_proxy_async();
+            mbar_expect_tx(&bars[b], Sh::TILE_BYTES);
+            tma_load_1d(sbuf + b * Sh::TILE_BYTES, in + tile * TILE, Sh::TILE_BYTES, &bars[b]);
+        }
+    };
+    // phase A on buffer b: per-row exclusive prefixes pre[], s_wex[b], s_agg[b]; publishes
+    // the aggregate (the inclusive prefix for tile 0)
+    unsigned par = 0u;  // bit b: mbarrier phase parity of buffer b
+    auto phase_a = [&](int b, int64_t tile, S (&pre)[R]) {
+        if ((tile + 1) * TILE <= n) {
+            mbar_wait(&bars[b], (par >> b) & 1u);
+            par ^= 1u << b;
+        }
+        S carry_w = SO::id();
+#pragma unroll
+        for (int q = 0; q < R; ++q) {
+            T x[VEC];
+            const int64_t p0 = load_row(b, tile, q, x);
+            int64_t r = SEG ? (p0 % L) : 0;
+            S run = SO::id();
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) run = SO::comb(run, lifted(x, p0, k, r));
+            S a = run;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const S o = SO::up(a, off);
+                if (lane >= off) a = SO::comb(o, a);
+            }
+            S ex = SO::up(a, 1);
+            if (lane == 0) ex = SO::id();
+            pre[q] = SO::comb(carry_w, ex);
+            carry_w = SO::comb(carry_w, SO::bcast(a, 31));
+        }
+        if (lane == 0) s_wtot[warp] = carry_w;
+        __syncthreads();
+        if (warp == 0) {
+            S a = lane < NW ? s_wtot[lane] : SO::id();
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const S o = SO::up(a, off);
+                if (lane >= off) a = SO::comb(o, a);
+            }
+            S wex = SO::up(a, 1);
+            if (lane == 0) wex = SO::id();
+            if (lane < NW) s_wex[b][lane] = wex;
+            const S agg = SO::bcast(a, NW - 1);
+            if (lane == 0) {
+                s_agg[b] = agg;
+                if (tile == 0) {
+                    S c0 = SO::id();
+                    if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+                    ts.publish(0, SO::comb(c0, agg), kStIncl);
+                } else {
+                    ts.publish(tile, agg, kStAgg);
+                }
+            }
+        }
+    };
+
+    S pre_cur[R], pre_nxt[R];
+    if (threadIdx.x == 0) {
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        fence_mbar_init();
+        const int64_t t0 = (int64_t)atomicAdd(counter, 1u);
+        s_tile[0] = t0;
+        issue(0, t0);
+    }
+    __syncthreads();
+    if (s_tile[0] >= ntiles) return;
+    phase_a(0, s_tile[0], pre_cur);
+    __syncthreads();
+
+    for (int it = 0;; ++it) {
+        const int b = it & 1;
+        const int64_t tile = s_tile[b];
+        if (tile >= ntiles) break;
+        // 1. next tile id + its TMA load
+        if (threadIdx.x == 0) {
+            const int64_t t1 = (int64_t)atomicAdd(counter, 1u);
+            s_tile[b ^ 1] = t1;
+            issue(b ^ 1, t1);
+        }
+        // 2. block-wide decoupled look-back for `tile`
+        S exc = SO::id();
+        if (tile == 0) {
+            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+        } else {
+            int64_t j = tile - 1;
+            while (true) {
+                const int64_t idx = j - threadIdx.x;
+                S v = SO::id();
+                unsigned st = kStIncl;
+                if (idx >= 0) {
+                    do {
+                        st = ts.poll(idx, v);
+                    } while (st == 0);
+                }
+                const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
+                if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
+                __syncthreads();
+                int kk = 1 << 20;
+#pragma unroll
+                for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
+                if ((int)threadIdx.x > kk || idx < 0) v = SO::id();
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const S o = SO::down(v, off);
+                    if (lane + off < 32) v = SO::comb(o, v);
+                }
+                if (lane == 0) s_lb_val[warp] = v;
+                __syncthreads();
+                S P = SO::id();
+#pragma unroll
+                for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_val[q]);
+                exc = SO::comb(P, exc);
+                __syncthreads();
+                if (kk < (1 << 20) || exc.f) break;
+                j -= kScanThreads;
+            }
+            if (threadIdx.x == 0) ts.publish(tile, SO::comb(exc, s_agg[b]), kStIncl);
+        }
+        if (threadIdx.x == 0) s_ex = exc;
+        __syncthreads();
+        // 3. next tile: local scan + publish its aggregate
+        const int64_t nt = s_tile[b ^ 1];
+        if (nt < ntiles) phase_a(b ^ 1, nt, pre_nxt);
+        // 4. write this tile
+        const S base = SO::comb(s_ex, s_wex[b][warp]);
+#pragma unroll
+        for (int q = 0; q < R; ++q) {
+            T x[VEC];
+            const int64_t p0 = load_row(b, tile, q, x);
+            S run = SO::comb(base, pre_cur[q]);
+            int64_t r = SEG ? (p0 % L) : 0;
+            T y[VEC];
+            int64_t yi[VEC];
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) {
+                run = SO::comb(run, lifted(x, p0, k, r));
+                y[k] = O::val(run.v);
+                yi[k] = O::idx(run.v);
+            }
+            if (p0 + VEC <= n) {
+                Vec16<T> w;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) w.e[k] = y[k];
+                int4 wv;
+                memcpy(&wv, &w, 16);
+                *reinterpret_cast<int4 *>(out + p0) = wv;
+            } else {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k)
+                    if (p0 + k < n) out[p0 + k] = y[k];
+            }
+            if (OP == kArgmin) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k)
+                    if (p0 + k < n) out_idx[p0 + k] = yi[k];
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < R; ++q) pre_cur[q] = pre_nxt[q];
+        __syncthreads();
+    }
+}
+
+// ws body: [0,256) tile counter | status words (8 B per tile) | aggs | incls
+static size_t scan_state_bytes(int64_t ntiles) { return align_up((size_t)ntiles * 8, 256); }
+
 template <int OP, typename T> struct ScanRun {
-    template <bool NN, bool SEG, bool AL>
+    template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
-                        int64_t *out_idx, const void *carry, const int64_t *carry_idx, void *ws, cudaStream_t st) {
-        using S = typename SOp<Op<OP, T>>::S;
-        const int64_t tile = (int64_t)kScanThreads * kScanRows * (16 / sizeof(T));
-        const int64_t ntiles = ceil_div(n, tile);
-        const ScanWs w = scan_ws_layout<S>(ws, ntiles);
-        if (cudaMemsetAsync(w.counter, 0, w.clear_bytes, st) != cudaSuccess) return FS_ERR_CUDA;
-        auto k = scan_lookback_kernel<OP, T, NN, SEG, AL>;
-        const int64_t cap = resident_blocks((const void *)k, kScanThreads);
+                        int64_t *out_idx, const void *carry, const int64_t *carry_idx, void *ws, bool aligned,
+                        cudaStream_t st) {
+        using Sh = ScanShape<OP, T>;
+        using S = typename SOp<Op<OP, T>, SEG>::S;
+        const int64_t ntiles = ceil_div(n, Sh::TILE);
+        char *b = (char *)ws + kWsHeader;
+        unsigned *counter = (unsigned *)b;
+        TileState<S, Sh::PACK> ts;
+        ts.w = (uint64_t *)(b + 256);
+        if constexpr (!Sh::PACK) {
+            ts.aggs = (S *)(b + 256 + scan_state_bytes(ntiles));
+            ts.incls = ts.aggs + ntiles;
+        }
+        if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntiles), st) != cudaSuccess) return FS_ERR_CUDA;
+        if constexpr (TMA && !NN) {
+            auto kp = scan_pipe_kernel<OP, T, SEG>;
+            const int smem = 2 * (int)Sh::TILE_BYTES;
+            static bool attr = false;
+            if (!attr) {
+                cudaFuncSetAttribute((const void *)kp, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                attr = true;
+            }
+            const int64_t cap = resident_blocks((const void *)kp, kScanThreads, smem);
+            const int64_t grid = ntiles < cap ? ntiles : cap;
+            kp<<<(unsigned)grid, kScanThreads, smem, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
+                                                           (const T *)carry, carry_idx, counter, ts, ntiles);
+            return launch_status();
+        }
+        auto k = scan_kernel<OP, T, NN, SEG, TMA>;
+        const int smem = TMA ? 2 * (int)Sh::TILE_BYTES : 0;
+        if (TMA) {
+            static bool attr = false;
+            if (!attr) {
+                cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                attr = true;
+            }
+        }
+        const int64_t cap = resident_blocks((const void *)k, kScanThreads, smem);
         const int64_t grid = ntiles < cap ? ntiles : cap;
-        k<<<(unsigned)grid, kScanThreads, 0, st>>>((const T *)in0, (const float *)in1, n, L, map.q0, map.q1,
-                                                   map.ibase, (T *)out, out_idx, (const T *)carry, carry_idx,
-                                                   w.counter, w.status, (S *)w.aggs, (S *)w.incls, ntiles);
+        k<<<(unsigned)grid, kScanThreads, smem, st>>>((const T *)in0, (const float *)in1, n, L, map.q0, map.q1,
+                                                      map.ibase, (T *)out, out_idx, (const T *)carry, carry_idx,
+                                                      counter, ts, ntiles, aligned);
         return launch_status();
     }
     static fs_status run(const fs_mapdesc *map, const void *in0, const void *in1, int64_t n, int64_t L, void *out,
@@ -310,26 +666,24 @@ template <int OP, typename T> struct ScanRun {
         bool al = ((uintptr_t)in0 & 15) == 0 && ((uintptr_t)out & 15) == 0;
         if (map->kind == FS_MAP_NN_DIST) {
             al = al && ((uintptr_t)in1 & 15) == 0;
-            if constexpr (sizeof(T) == 4) {
-                if (al) return go<true, false, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
-                return go<true, false, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
-            }
+            if constexpr (sizeof(T) == 4)
+                return go<true, false, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
             return FS_ERR_UNSUPPORTED;
         }
         if (seg) {
-            if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
-            return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
+            if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
+            return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
         }
-        if (al) return go<false, false, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
-        return go<false, false, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, st);
+        if (al) return go<false, false, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
+        return go<false, false, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
     }
 };
 
 size_t scan_ws(int op, int dt, int64_t n) {
-    const int64_t tile = (int64_t)kScanThreads * kScanRows * (16 / (int64_t)dtype_size(dt));
+    const int R = (op != FS_ARGMIN && dtype_size(dt) == 4) ? 8 : 4;
+    const int64_t tile = (int64_t)kScanThreads * R * (16 / (int64_t)dtype_size(dt));
     const int64_t ntiles = ceil_div(n, tile);
-    const size_t s = align_up(acc_size(op, dt) + 4, 8);  // S = {V, int}, padded
-    return kWsHeader + 256 + align_up((size_t)ntiles * 4, 256) + 2 * align_up((size_t)ntiles * (s + 8), 256);
+    return kWsHeader + 256 + scan_state_bytes(ntiles) + 2 * align_up((size_t)ntiles * 32, 256);
 }
 
 fs_status scan_run(int op, int dt, const fs_mapdesc &map, const void *in0, const void *in1, int64_t n, int64_t L,
