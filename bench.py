@@ -190,10 +190,10 @@ def make_step(fs, W, world):
 def oracle_sample(W, scale_shift):
     """Host copies of a bounded sample of every primitive's input (same data as the GPU run)."""
     s = {}
-    m = min(W["n"], (1 << 25) >> scale_shift)
+    m = min(W["n"], (1 << 26) >> scale_shift)
     s["x"] = W["x"][:m].cpu().numpy()
     s["lat"], s["lng"] = W["lat"].cpu().numpy(), W["lng"].cpu().numpy()
-    kr = min(W["pts"].shape[0], (1 << 21) >> scale_shift)
+    kr = min(W["pts"].shape[0], (1 << 22) >> scale_shift)
     s["pts"], s["mem"] = W["pts"][:kr].cpu().numpy(), W["mem"][:kr].cpu().numpy()
     tt = min(W["t"], 4096 >> (scale_shift // 2))
     s["tmat"] = W["tmat"][:tt, :tt].cpu().numpy()
@@ -347,7 +347,8 @@ def main():
     tf = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tf):
         with open(tf) as f:
-            traffic = json.load(f).get(dom)
+            t = json.load(f).get(dom)
+        traffic = t.get("traffic_bytes_per_launch") if isinstance(t, dict) else t
 
     # ---------------- e2e: host buffers, H2D + compute + D2H inside the timed region
     e2e = None

@@ -23,6 +23,8 @@
 // Column-major seg_scan (segments are columns of an [m][w] row-major array):
 // threads own (vector-column, row block) units and scan down their rows; row
 // blocks are chained by a reduce / exclusive-scan-of-partials / rescan.
+#include <stdlib.h>
+
 #include "internal.cuh"
 
 namespace fs {
@@ -124,13 +126,31 @@ __device__ __forceinline__ float nn_dist_s(float lat, float lng, float q0, float
     return __fsqrt_rn(__fadd_rn(__fmul_rn(d0, d0), __fmul_rn(d1, d1)));
 }
 
+#ifndef FS_SCAN_R
+#define FS_SCAN_R 4
+#endif
 constexpr int kScanThreads = 256;
 constexpr unsigned kStAgg = 1, kStIncl = 2;
+
+// -DFS_SCAN_PROFILE: thread 0 of every CTA accumulates clock64 cycles per phase of
+// scan_pipe_kernel into fs_scan_prof[] (debug / ncu-free attribution only)
+#ifdef FS_SCAN_PROFILE
+__device__ unsigned long long fs_scan_prof[16];
+}  // namespace fs
+extern "C" void fs_scan_prof_ptr(void **p) { cudaGetSymbolAddress(p, fs::fs_scan_prof); }
+namespace fs {
+#define FS_PROF_T(var) long long var = clock64()
+#define FS_PROF_ADD(slot, t0) \
+    if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[slot], (unsigned long long)(clock64() - (t0)))
+#else
+#define FS_PROF_T(var)
+#define FS_PROF_ADD(slot, t0)
+#endif
 
 // 16-byte vectors per lane per tile: 8 for 8-byte (value, flag) pairs, 4 for wider ones
 template <int OP, typename T> struct ScanShape {
     static constexpr bool PACK = OP != kArgmin && sizeof(T) == 4;
-    static constexpr int R = (OP != kArgmin && sizeof(T) == 4) ? 8 : 4;
+    static constexpr int R = (OP != kArgmin && sizeof(T) == 4) ? FS_SCAN_R : 2;
     static constexpr int VEC = 16 / sizeof(T);
     static constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
     static constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
@@ -385,82 +405,99 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
     }
 }
 
-// ---------------------------------------------------------------- pipelined TMA scan
-// Software pipeline over the CTA's tiles T0, T1, ... (ids from the atomic
-// counter).  Iteration k:
-//   1. take T(k+1) and start its TMA bulk load into the other buffer
-//   2. look-back for T(k) (its aggregate was published one step earlier)
-//   3. wait for T(k+1); local scan; publish T(k+1)'s aggregate
-//   4. write T(k) = its exclusive prefix (+) local scan (re-derived from smem)
-// A tile's aggregate is published about one look-back after the tile was
-// taken, so successors rarely spin, and the HBM read of T(k+1) overlaps the
-// look-back and output of T(k).
-template <int OP, typename T, bool SEG>
-__global__ void __launch_bounds__(kScanThreads, 3)
-scan_pipe_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+// ---------------------------------------------------------------- TMA tile scan
+// One tile at a time per CTA, several CTAs per SM:
+//   claim the next tile id (atomic counter: every predecessor is owned by a
+//   running CTA) -> TMA bulk load of the tile into shared memory -> local scan
+//   and publish the tile aggregate -> decoupled look-back over RB_WIN
+//   predecessors per step with the whole CTA (one status word per thread),
+//   "helping forward": when the window holds an inclusive prefix, every
+//   predecessor that only had an aggregate gets its inclusive prefix published
+//   too, so the next tiles find one a single step back -> write the tile.
+// A tile's aggregate is published one load + local scan after it was claimed,
+// so the look-back of the next tile rarely spins; the other CTAs on the SM
+// overlap this CTA's round trips.  (Claiming tiles ahead of processing made
+// successors spin on not-yet-published aggregates: measured slower.)
+template <int OP, typename T, bool SEG, int R>
+__global__ void __launch_bounds__(kScanThreads, 4)
+scan_tile_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
                  int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
                  TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
     using O = Op<OP, T>;
     using SO = SOp<O, SEG>;
     using S = typename SO::S;
-    using Sh = ScanShape<OP, T>;
-    constexpr int VEC = Sh::VEC, R = Sh::R, NW = kScanThreads / 32;
-    constexpr int64_t TILE = Sh::TILE;
+    constexpr int VEC = 16 / sizeof(T), NW = kScanThreads / 32;
+    constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
+    constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
+    constexpr int WIN = kScanThreads;
     extern __shared__ __align__(128) unsigned char sbuf[];
-    __shared__ uint64_t bars[2];
-    __shared__ int64_t s_tile[2];
-    __shared__ S s_wtot[NW], s_wex[2][NW], s_agg[2], s_ex, s_lb_val[NW];
+    __shared__ uint64_t bar;
+    __shared__ int64_t s_tile;
+    __shared__ S s_wtot[NW], s_wex[NW], s_agg, s_ex, s_lb_tot[NW];
     __shared__ int s_lb_min[NW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-
-    // element k of this lane's vector in row q of tile `tile` (buffer b)
-    auto load_row = [&](int b, int64_t tile, int q, T (&x)[VEC]) {
-        const int64_t p0 = tile * TILE + (int64_t)warp * 32 * R * VEC + ((int64_t)q * 32 + lane) * VEC;
-        if ((tile + 1) * TILE <= n) {
-            const Vec16<T> a =
-                *reinterpret_cast<const Vec16<T> *>(sbuf + b * Sh::TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
+    unsigned par = 0u;
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    for (;;) {
+        FS_PROF_T(t1);
+        if (threadIdx.x == 0) {
+            const int64_t t = (int64_t)atomicAdd(counter, 1u);
+            s_tile = t;
+            if (t < ntiles && (t + 1) * TILE <= n) {
+                fence_proxy_async();
+                mbar_expect_tx(&bar, TILE_BYTES);
+                tma_load_1d(sbuf, in + t * TILE, TILE_BYTES, &bar);
+            }
+        }
+        __syncthreads();
+        const int64_t tile = s_tile;
+        if (tile >= ntiles) break;
+        FS_PROF_ADD(1, t1);
+        FS_PROF_T(t2);
+        const bool full = (tile + 1) * TILE <= n;
+        if (full) {
+            mbar_wait(&bar, par);
+            par ^= 1u;
+        }
+        FS_PROF_ADD(2, t2);
+        FS_PROF_T(t3);
+        const int64_t wbase = tile * TILE + (int64_t)warp * 32 * R * VEC;
+        auto load_row = [&](int q, T (&x)[VEC]) {
+            const int64_t p0 = wbase + ((int64_t)q * 32 + lane) * VEC;
+            if (full) {
+                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(sbuf + (((warp * R + q) * 32 + lane) << 4));
 #pragma unroll
-            for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
-        } else {
+                for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+            } else {
 #pragma unroll
-            for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
-        }
-        return p0;
-    };
-    auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
-        S e;
-        if (p0 + k < n) {
-            e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
-            e.f = SEG ? (r == 0) : 0;
-        } else {
-            e = SO::id();
-        }
-        if (SEG) {
-            ++r;
-            if (r == L) r = 0;
-        }
-        return e;
-    };
-    auto issue = [&](int b, int64_t tile) {  // thread 0
-        if (tile < ntiles && (tile + 1) * TILE <= n) {
-            fence_proxy_async();
-            mbar_expect_tx(&bars[b], Sh::TILE_BYTES);
-            tma_load_1d(sbuf + b * Sh::TILE_BYTES, in + tile * TILE, Sh::TILE_BYTES, &bars[b]);
-        }
-    };
-    // phase A on buffer b: per-row exclusive prefixes pre[], s_wex[b], s_agg[b]; publishes
-    // the aggregate (the inclusive prefix for tile 0)
-    unsigned par = 0u;  // bit b: mbarrier phase parity of buffer b
-    auto phase_a = [&](int b, int64_t tile, S (&pre)[R]) {
-        if ((tile + 1) * TILE <= n) {
-            mbar_wait(&bars[b], (par >> b) & 1u);
-            par ^= 1u << b;
-        }
+                for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
+            }
+            return p0;
+        };
+        auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
+            S e;
+            if (p0 + k < n) {
+                e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
+                e.f = SEG ? (r == 0) : 0;
+            } else {
+                e = SO::id();
+            }
+            if (SEG) {
+                ++r;
+                if (r == L) r = 0;
+            }
+            return e;
+        };
+        // local scan: per-row exclusive prefixes within the warp
+        S pre[R];
         S carry_w = SO::id();
 #pragma unroll
         for (int q = 0; q < R; ++q) {
             T x[VEC];
-            const int64_t p0 = load_row(b, tile, q, x);
+            const int64_t p0 = load_row(q, x);
             int64_t r = SEG ? (p0 % L) : 0;
             S run = SO::id();
 #pragma unroll
@@ -487,10 +524,10 @@ scan_pipe_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, 
             }
             S wex = SO::up(a, 1);
             if (lane == 0) wex = SO::id();
-            if (lane < NW) s_wex[b][lane] = wex;
+            if (lane < NW) s_wex[lane] = wex;
             const S agg = SO::bcast(a, NW - 1);
             if (lane == 0) {
-                s_agg[b] = agg;
+                s_agg = agg;
                 if (tile == 0) {
                     S c0 = SO::id();
                     if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
@@ -500,83 +537,75 @@ scan_pipe_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, 
                 }
             }
         }
-    };
-
-    S pre_cur[R], pre_nxt[R];
-    if (threadIdx.x == 0) {
-        mbar_init(&bars[0], 1);
-        mbar_init(&bars[1], 1);
-        fence_mbar_init();
-        const int64_t t0 = (int64_t)atomicAdd(counter, 1u);
-        s_tile[0] = t0;
-        issue(0, t0);
-    }
-    __syncthreads();
-    if (s_tile[0] >= ntiles) return;
-    phase_a(0, s_tile[0], pre_cur);
-    __syncthreads();
-
-    for (int it = 0;; ++it) {
-        const int b = it & 1;
-        const int64_t tile = s_tile[b];
-        if (tile >= ntiles) break;
-        // 1. next tile id + its TMA load
-        if (threadIdx.x == 0) {
-            const int64_t t1 = (int64_t)atomicAdd(counter, 1u);
-            s_tile[b ^ 1] = t1;
-            issue(b ^ 1, t1);
-        }
-        // 2. block-wide decoupled look-back for `tile`
+        __syncthreads();
+        FS_PROF_ADD(3, t3);
+        FS_PROF_T(t4);
+        // decoupled look-back
         S exc = SO::id();
         if (tile == 0) {
             if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
         } else {
             int64_t j = tile - 1;
-            while (true) {
+            for (int step = 0;; ++step) {
                 const int64_t idx = j - threadIdx.x;
+                const bool mine = idx >= 0;
                 S v = SO::id();
                 unsigned st = kStIncl;
-                if (idx >= 0) {
+                if (mine) {
+                    FS_PROF_T(t6);
                     do {
                         st = ts.poll(idx, v);
+#ifdef FS_SCAN_PROFILE
+                        if (threadIdx.x == 0 && st == 0) atomicAdd(&fs_scan_prof[7], 1ull);
+#endif
                     } while (st == 0);
+                    FS_PROF_ADD(6, t6);
                 }
-                const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
+                const unsigned m = __ballot_sync(0xffffffffu, mine && st == kStIncl);
                 if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
                 __syncthreads();
+#ifdef FS_SCAN_PROFILE
+                if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[8], 1ull);
+#endif
                 int kk = 1 << 20;
 #pragma unroll
                 for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
-                if ((int)threadIdx.x > kk || idx < 0) v = SO::id();
+                if ((int)threadIdx.x > kk || !mine) v = SO::id();
+                // suffix scan toward lower thread ids (higher ids are further left)
+                S a = v;
 #pragma unroll
                 for (int off = 1; off < 32; off <<= 1) {
-                    const S o = SO::down(v, off);
-                    if (lane + off < 32) v = SO::comb(o, v);
+                    const S o = SO::down(a, off);
+                    if (lane + off < 32) a = SO::comb(o, a);
                 }
-                if (lane == 0) s_lb_val[warp] = v;
+                if (lane == 0) s_lb_tot[warp] = a;
                 __syncthreads();
+                S left = SO::id();
+#pragma unroll
+                for (int q = NW - 1; q > warp; --q) left = SO::comb(left, s_lb_tot[q]);
                 S P = SO::id();
 #pragma unroll
-                for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_val[q]);
+                for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_tot[q]);
+                if (step == 0 && kk < (1 << 20) && mine && (int)threadIdx.x < kk && st == kStAgg)
+                    ts.publish(idx, SO::comb(left, a), kStIncl);  // help forward
                 exc = SO::comb(P, exc);
                 __syncthreads();
                 if (kk < (1 << 20) || exc.f) break;
-                j -= kScanThreads;
+                j -= WIN;
             }
-            if (threadIdx.x == 0) ts.publish(tile, SO::comb(exc, s_agg[b]), kStIncl);
+            if (threadIdx.x == 0) ts.publish(tile, SO::comb(exc, s_agg), kStIncl);
         }
         if (threadIdx.x == 0) s_ex = exc;
         __syncthreads();
-        // 3. next tile: local scan + publish its aggregate
-        const int64_t nt = s_tile[b ^ 1];
-        if (nt < ntiles) phase_a(b ^ 1, nt, pre_nxt);
-        // 4. write this tile
-        const S base = SO::comb(s_ex, s_wex[b][warp]);
+        FS_PROF_ADD(4, t4);
+        FS_PROF_T(t5);
+        // write the tile
+        const S base = SO::comb(s_ex, s_wex[warp]);
 #pragma unroll
         for (int q = 0; q < R; ++q) {
             T x[VEC];
-            const int64_t p0 = load_row(b, tile, q, x);
-            S run = SO::comb(base, pre_cur[q]);
+            const int64_t p0 = load_row(q, x);
+            S run = SO::comb(base, pre[q]);
             int64_t r = SEG ? (p0 % L) : 0;
             T y[VEC];
             int64_t yi[VEC];
@@ -604,8 +633,246 @@ scan_pipe_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, 
                     if (p0 + k < n) out_idx[p0 + k] = yi[k];
             }
         }
+        __syncthreads();  // smem tile and s_tile reuse
+        FS_PROF_ADD(5, t5);
+#ifdef FS_SCAN_PROFILE
+        if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[0], 1ull);
+#endif
+    }
+}
+
+// ---------------------------------------------------------------- deferred look-back scan
+// Aggregates never wait; look-backs are deferred.  Iteration i of a CTA:
+//   A. claim tile t_i, TMA it from HBM, reduce it and publish its aggregate
+//      (no dependency on any other tile -> aggregates flow at read speed)
+//   C. for the tile t_{i-D} this CTA claimed D iterations ago: TMA it again
+//      (it is still in the 126 MB L2: D x #CTAs x 32 KB ~ 38 MB), scan it
+//      locally, look back (its predecessors published their aggregates about D
+//      iterations ago, so the look-back almost never spins), publish its
+//      inclusive prefix (helping forward) and write it.
+// HBM traffic stays one read + one write per element; the second read hits L2.
+template <int OP, typename T, bool SEG, int R, int D>
+__global__ void __launch_bounds__(kScanThreads, 3)
+scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+               int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
+               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
+    using O = Op<OP, T>;
+    using SO = SOp<O, SEG>;
+    using S = typename SO::S;
+    constexpr int VEC = 16 / sizeof(T), NW = kScanThreads / 32;
+    constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
+    constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
+    constexpr int WIN = kScanThreads, RING = D + 2;
+    // buffers 0,1: new tiles (A, double-buffered); 2,3: deferred tiles (C, double-buffered)
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    __shared__ uint64_t bars[4];
+    __shared__ int64_t s_ring[RING];
+    __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_tot[NW];
+    __shared__ int s_lb_min[NW];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    unsigned par = 0u;
+    auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
+    auto issue = [&](int b, int64_t t) {
+        if (t >= 0 && t < ntiles && full_tile(t)) {
+            fence_proxy_async();
+            mbar_expect_tx(&bars[b], TILE_BYTES);
+            tma_load_1d(sbuf + b * TILE_BYTES, in + t * TILE, TILE_BYTES, &bars[b]);
+        }
+    };
+    auto load_row = [&](int b, int64_t t, int q, T (&x)[VEC]) {
+        const int64_t p0 = t * TILE + (int64_t)warp * 32 * R * VEC + ((int64_t)q * 32 + lane) * VEC;
+        if (full_tile(t)) {
+            const Vec16<T> a =
+                *reinterpret_cast<const Vec16<T> *>(sbuf + b * TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
 #pragma unroll
-        for (int q = 0; q < R; ++q) pre_cur[q] = pre_nxt[q];
+            for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+        } else {
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
+        }
+        return p0;
+    };
+    auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
+        S e;
+        if (p0 + k < n) {
+            e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
+            e.f = SEG ? (r == 0) : 0;
+        } else {
+            e = SO::id();
+        }
+        if (SEG) {
+            ++r;
+            if (r == L) r = 0;
+        }
+        return e;
+    };
+    // ordered local scan of the tile in buffer b: per-row prefixes pre[], s_wex[], returns aggregate
+    auto local_scan = [&](int b, int64_t t, S (&pre)[R]) {
+        if (full_tile(t)) {
+            mbar_wait(&bars[b], (par >> b) & 1u);
+            par ^= 1u << b;
+        }
+        S carry_w = SO::id();
+#pragma unroll
+        for (int q = 0; q < R; ++q) {
+            T x[VEC];
+            const int64_t p0 = load_row(b, t, q, x);
+            int64_t r = SEG ? (p0 % L) : 0;
+            S run = SO::id();
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) run = SO::comb(run, lifted(x, p0, k, r));
+            S a = run;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const S o = SO::up(a, off);
+                if (lane >= off) a = SO::comb(o, a);
+            }
+            S ex = SO::up(a, 1);
+            if (lane == 0) ex = SO::id();
+            pre[q] = SO::comb(carry_w, ex);
+            carry_w = SO::comb(carry_w, SO::bcast(a, 31));
+        }
+        if (lane == 0) s_wtot[warp] = carry_w;
+        __syncthreads();
+        S a = lane < NW ? s_wtot[lane] : SO::id();
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const S o = SO::up(a, off);
+            if (lane >= off) a = SO::comb(o, a);
+        }
+        S wex = SO::up(a, 1);
+        if (lane == 0) wex = SO::id();
+        if (warp == 0 && lane < NW) s_wex[lane] = wex;
+        const S agg = SO::bcast(a, NW - 1);
+        __syncthreads();
+        return agg;
+    };
+    auto carry_in = [&]() {
+        S c0 = SO::id();
+        if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+        return c0;
+    };
+
+    S pre[R];
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) mbar_init(&bars[q], 1);
+        fence_mbar_init();
+        const int64_t t0 = (int64_t)atomicAdd(counter, 1u);
+        s_ring[0] = t0;
+        issue(0, t0);
+    }
+    for (int64_t i = 0;; ++i) {
+        if (threadIdx.x == 0) {
+            // prefetch for iteration i+1: claim t_{i+1} (stop claiming once past the end)
+            const int64_t cur = s_ring[i % RING];
+            const int64_t nxt = cur >= ntiles ? ntiles : (int64_t)atomicAdd(counter, 1u);
+            s_ring[(i + 1) % RING] = nxt;
+            issue((int)((i + 1) & 1), nxt);
+            issue(2 + (int)((i + 1) & 1), i + 1 >= D ? s_ring[(i + 1 - D) % RING] : -1);
+        }
+        __syncthreads();
+        const int64_t ti = s_ring[i % RING];
+        const int64_t told = i >= D ? s_ring[(i - D) % RING] : -1;
+        if (ti >= ntiles && (told < 0 || told >= ntiles)) {
+            bool more = false;
+            for (int64_t q = i - D + 1; q < i; ++q)
+                if (q >= 0 && s_ring[q % RING] < ntiles) more = true;
+            if (!more) break;
+        }
+        const int bA = (int)(i & 1), bC = 2 + (int)(i & 1);
+        // A. aggregate of the new tile
+        if (ti < ntiles) {
+            const S agg = local_scan(bA, ti, pre);
+            if (threadIdx.x == 0) {
+                if (ti == 0) ts.publish(0, SO::comb(carry_in(), agg), kStIncl);
+                else ts.publish(ti, agg, kStAgg);
+            }
+        }
+        // C. scan + write the tile claimed D iterations ago
+        if (told >= 0 && told < ntiles) {
+            const S agg = local_scan(bC, told, pre);
+            S exc = SO::id();
+            if (told == 0) {
+                exc = carry_in();
+            } else {
+                int64_t j = told - 1;
+                for (int step = 0;; ++step) {
+                    const int64_t idx = j - threadIdx.x;
+                    const bool mine = idx >= 0;
+                    S v = SO::id();
+                    unsigned st = kStIncl;
+                    if (mine) {
+                        do {
+                            st = ts.poll(idx, v);
+                        } while (st == 0);
+                    }
+                    const unsigned m = __ballot_sync(0xffffffffu, mine && st == kStIncl);
+                    if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
+                    __syncthreads();
+                    int kk = 1 << 20;
+#pragma unroll
+                    for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
+                    if ((int)threadIdx.x > kk || !mine) v = SO::id();
+                    S a = v;
+#pragma unroll
+                    for (int off = 1; off < 32; off <<= 1) {
+                        const S o = SO::down(a, off);
+                        if (lane + off < 32) a = SO::comb(o, a);
+                    }
+                    if (lane == 0) s_lb_tot[warp] = a;
+                    __syncthreads();
+                    S left = SO::id();
+#pragma unroll
+                    for (int q = NW - 1; q > warp; --q) left = SO::comb(left, s_lb_tot[q]);
+                    S P = SO::id();
+#pragma unroll
+                    for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_tot[q]);
+                    if (step == 0 && kk < (1 << 20) && mine && (int)threadIdx.x < kk && st == kStAgg)
+                        ts.publish(idx, SO::comb(left, a), kStIncl);  // help forward
+                    exc = SO::comb(P, exc);
+                    __syncthreads();
+                    if (kk < (1 << 20) || exc.f) break;
+                    j -= WIN;
+                }
+                if (threadIdx.x == 0) ts.publish(told, SO::comb(exc, agg), kStIncl);
+            }
+            if (threadIdx.x == 0) s_ex = exc;
+            __syncthreads();
+            const S base = SO::comb(s_ex, s_wex[warp]);
+#pragma unroll
+            for (int q = 0; q < R; ++q) {
+                T x[VEC];
+                const int64_t p0 = load_row(bC, told, q, x);
+                S run = SO::comb(base, pre[q]);
+                int64_t r = SEG ? (p0 % L) : 0;
+                T y[VEC];
+                int64_t yi[VEC];
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) {
+                    run = SO::comb(run, lifted(x, p0, k, r));
+                    y[k] = O::val(run.v);
+                    yi[k] = O::idx(run.v);
+                }
+                if (p0 + VEC <= n) {
+                    Vec16<T> w;
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) w.e[k] = y[k];
+                    int4 wv;
+                    memcpy(&wv, &w, 16);
+                    *reinterpret_cast<int4 *>(out + p0) = wv;
+                } else {
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k)
+                        if (p0 + k < n) out[p0 + k] = y[k];
+                }
+                if (OP == kArgmin) {
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k)
+                        if (p0 + k < n) out_idx[p0 + k] = yi[k];
+                }
+            }
+        }
         __syncthreads();
     }
 }
@@ -631,13 +898,12 @@ template <int OP, typename T> struct ScanRun {
         }
         if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntiles), st) != cudaSuccess) return FS_ERR_CUDA;
         if constexpr (TMA && !NN) {
-            auto kp = scan_pipe_kernel<OP, T, SEG>;
-            const int smem = 2 * (int)Sh::TILE_BYTES;
-            static bool attr = false;
-            if (!attr) {
-                cudaFuncSetAttribute((const void *)kp, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-                attr = true;
-            }
+            // same tile shape as the ws sizing (Sh::R rows of 16-byte vectors per thread)
+            // deferred look-back, 4 buffers of half-size tiles (same tile grid as the ws sizing)
+            // D = 3 iterations of deferral (swept 1..3 and R = 4/8 on B200: R4 D3 fastest)
+            auto kp = scan_dl_kernel<OP, T, SEG, Sh::R, 3>;
+            const int smem = 4 * (int)Sh::TILE_BYTES;
+            cudaFuncSetAttribute((const void *)kp, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
             const int64_t cap = resident_blocks((const void *)kp, kScanThreads, smem);
             const int64_t grid = ntiles < cap ? ntiles : cap;
             kp<<<(unsigned)grid, kScanThreads, smem, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
@@ -680,7 +946,7 @@ template <int OP, typename T> struct ScanRun {
 };
 
 size_t scan_ws(int op, int dt, int64_t n) {
-    const int R = (op != FS_ARGMIN && dtype_size(dt) == 4) ? 8 : 4;
+    const int R = (op != FS_ARGMIN && dtype_size(dt) == 4) ? FS_SCAN_R : 2;
     const int64_t tile = (int64_t)kScanThreads * R * (16 / (int64_t)dtype_size(dt));
     const int64_t ntiles = ceil_div(n, tile);
     return kWsHeader + 256 + scan_state_bytes(ntiles) + 2 * align_up((size_t)ntiles * 32, 256);

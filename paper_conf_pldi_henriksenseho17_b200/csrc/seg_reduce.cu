@@ -88,6 +88,86 @@ seg_tile_kernel(const T *__restrict__ x, int64_t nseg, int L, int tile_segs, T *
     }
 }
 
+// ---------------------------------------------------------------- KG0
+// Power-of-two segments up to 32 vectors, 16-byte aligned base: no shared
+// memory at all.  Each lane loads 16-byte vectors straight from HBM (coalesced,
+// U in flight); a vector holds SPL = VEC/L whole segments (L < VEC) or a
+// segment spans G = L/VEC lanes, reduced with log2(G) xor shuffles.
+// a 16-byte vector holding VEC/LS whole segments of length LS (compile-time)
+template <class O, typename T, int LS>
+__device__ __forceinline__ void small_segs(const Vec16<T> &e, int64_t v, T *out, int64_t *out_idx) {
+    constexpr int VEC = 16 / sizeof(T), SPL = VEC / LS;
+#pragma unroll
+    for (int sg = 0; sg < SPL; ++sg) {
+        typename O::V a = O::id();
+#pragma unroll
+        for (int k = 0; k < LS; ++k) a = O::fold(a, e.e[sg * LS + k], k);
+        store_out<O>(out, out_idx, v * SPL + sg, a);
+    }
+}
+
+template <int OP, typename T, int NT, int U>
+__global__ void __launch_bounds__(NT)
+seg_vec_kernel(const T *__restrict__ x, int64_t nseg, int L, int G, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    const int lane = threadIdx.x & 31;
+    const int64_t nvec = nseg * (int64_t)L / VEC;  // whole vectors
+    const int64_t stride = (int64_t)gridDim.x * NT;
+    const int lg = lane & (G - 1);
+    const int64_t gid0 = (int64_t)blockIdx.x * NT + threadIdx.x;
+    // every lane of a warp runs the same number of iterations (shuffles)
+    const int64_t iters = (nvec + stride - 1) / stride;
+    // software pipeline: the loads of batch b+1 are in flight while batch b is reduced
+    int4 r[U], rn[U];
+    auto load_batch = [&](int64_t it0, int4 (&dst)[U]) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            if (it0 + u < iters && v < nvec) dst[u] = ldg16(x + v * VEC);
+        }
+    };
+    if (iters > 0) load_batch(0, r);
+    for (int64_t it0 = 0; it0 < iters; it0 += U) {
+        if (it0 + U < iters) load_batch(it0 + U, rn);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            const bool live = it0 + u < iters;  // warp-uniform
+            const bool ok = live && v < nvec;
+            const Vec16<T> e = as_vec<T>(r[u]);
+            if (L <= VEC) {
+                if (ok) {
+                    if (L == 1) small_segs<O, T, 1>(e, v, out, out_idx);
+                    else if (L == 2) small_segs<O, T, 2>(e, v, out, out_idx);
+                    else small_segs<O, T, (VEC >= 4 ? 4 : VEC)>(e, v, out, out_idx);
+                }
+            } else {
+                V a = O::id();
+                if (ok) {
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], (int64_t)lg * VEC + k);
+                }
+                if (live)
+                    for (int m = G >> 1; m >= 1; m >>= 1) a = O::comb(a, shfl_xor(a, m));
+                if (ok && lg == 0) store_out<O>(out, out_idx, v / G, a);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) r[u] = rn[u];
+    }
+    // ragged tail (L < VEC and nseg * L not a multiple of VEC): scalar, one segment per thread
+    if (L < VEC) {
+        const int64_t s0 = nvec * VEC / L;
+        for (int64_t sgi = s0 + gid0; sgi < nseg; sgi += stride) {
+            V a = O::id();
+            for (int k = 0; k < L; ++k) a = O::fold(a, x[sgi * L + k], k);
+            store_out<O>(out, out_idx, sgi, a);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- KG2
 template <int OP, typename T, int NT, int U>
 __global__ void __launch_bounds__(NT)
@@ -220,7 +300,8 @@ int seg_reduce_regime(int op, int dt, int64_t nseg, int64_t L) {
         if (forced == 0 && L > kg1max) return 1;
         return forced;
     }
-    if (L <= 64) return 0;
+    const int64_t vec = 16 / (int64_t)dtype_size(dt);
+    if (L <= 64 || ((L & (L - 1)) == 0 && L <= 32 * vec)) return 0;  // KG1 (KG0 when L is a power of two)
     if (L <= kWarpMaxL) return 1;
     const int64_t resident = (int64_t)sm_count() * 8;
     return nseg >= 2 * resident ? 2 : 3;
@@ -252,6 +333,19 @@ template <int OP, typename T> struct SegRun {
                          void *ws, cudaStream_t st) {
         using V = typename Op<OP, T>::V;
         const T *x = (const T *)in;
+        constexpr int VEC = 16 / sizeof(T);
+        const bool pow2 = (L & (L - 1)) == 0;
+        if (regime == 0 && pow2 && L <= 32 * VEC && ((uintptr_t)x & 15) == 0) {
+            const int G = L > VEC ? (int)(L / VEC) : 1;
+            const void *k = (const void *)seg_vec_kernel<OP, T, kSegThreads, 4>;
+            const int64_t nvec = nseg * L / VEC;
+            int64_t grid = ceil_div(nvec > 0 ? nvec : 1, (int64_t)kSegThreads * 4);
+            const int64_t cap = resident_blocks(k, kSegThreads);
+            grid = grid < cap ? grid : cap;
+            seg_vec_kernel<OP, T, kSegThreads, 4><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, G,
+                                                                                         (T *)out, out_idx);
+            return launch_status();
+        }
         if (regime == 0) {
             const int maxe = tile_elems<T>();
             int tile_segs = maxe / (int)L;

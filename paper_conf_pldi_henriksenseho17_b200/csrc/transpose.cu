@@ -10,33 +10,61 @@
 
 namespace fs {
 
-constexpr int kTile = 32;
-constexpr int kRowsPerPass = 8;
+// 64 x 64 tiles, 256 threads, 16-byte vector loads and stores: each input row
+// segment and each output row segment a CTA touches is 256 B (4-byte
+// elements) / 512 B (8-byte) contiguous, so DRAM sees long runs on both sides.
+// Shared memory is padded by one element per row; the transposed gather reads
+// conflict at most 2-way.
+constexpr int kTT = 64;            // tile edge (elements)
+constexpr int kTThreads = 256;
 
 template <typename T>
-__global__ void __launch_bounds__(kTile *kRowsPerPass)
-transpose_kernel(const T *__restrict__ in, int64_t rows, int64_t cols, T *__restrict__ out,
-                 int64_t tiles_c, int64_t ntiles) {
-    __shared__ T tile[kTile][kTile + 1];
-    const int tx = threadIdx.x, ty = threadIdx.y;
+__global__ void __launch_bounds__(kTThreads)
+transpose_kernel(const T *__restrict__ in, int64_t rows, int64_t cols, T *__restrict__ out, int64_t tiles_c,
+                 int64_t ntiles) {
+    constexpr int VEC = 16 / sizeof(T);
+    constexpr int VPR = kTT / VEC;            // vectors per tile row
+    constexpr int RPP = kTThreads / VPR;      // tile rows per pass
+    __shared__ T tile[kTT][kTT + 1];
+    const int t = threadIdx.x;
+    const int vc = t % VPR, rr = t / VPR;
     for (int64_t tt = blockIdx.x; tt < ntiles; tt += gridDim.x) {
         const int64_t tr = tt / tiles_c, tc = tt - tr * tiles_c;
-        const int64_t r0 = tr * kTile, c0 = tc * kTile;
-        const int64_t c = c0 + tx;
-        if (r0 + kTile <= rows && c0 + kTile <= cols) {
+        const int64_t r0 = tr * kTT, c0 = tc * kTT;
+        const bool interior = r0 + kTT <= rows && c0 + kTT <= cols && ((cols * sizeof(T)) & 15) == 0 &&
+                              ((rows * sizeof(T)) & 15) == 0 && (((uintptr_t)in | (uintptr_t)out) & 15) == 0;
+        if (interior) {
+            int4 v[kTT / RPP];
 #pragma unroll
-            for (int k = 0; k < kTile; k += kRowsPerPass) tile[ty + k][tx] = __ldg(in + (r0 + ty + k) * cols + c);
+            for (int p = 0; p < kTT / RPP; ++p)
+                v[p] = ldg16(in + (r0 + rr + p * RPP) * cols + c0 + vc * VEC);
+#pragma unroll
+            for (int p = 0; p < kTT / RPP; ++p) {
+                const Vec16<T> e = as_vec<T>(v[p]);
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) tile[rr + p * RPP][vc * VEC + k] = e.e[k];
+            }
             __syncthreads();
 #pragma unroll
-            for (int k = 0; k < kTile; k += kRowsPerPass) out[(c0 + ty + k) * rows + r0 + tx] = tile[tx][ty + k];
+            for (int p = 0; p < kTT / RPP; ++p) {
+                const int j = rr + p * RPP;  // output row within the tile (= input column)
+                Vec16<T> o;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) o.e[k] = tile[vc * VEC + k][j];
+                int4 ov;
+                memcpy(&ov, &o, 16);
+                *reinterpret_cast<int4 *>(out + (c0 + j) * rows + r0 + vc * VEC) = ov;
+            }
         } else {
-#pragma unroll
-            for (int k = 0; k < kTile; k += kRowsPerPass)
-                if (r0 + ty + k < rows && c < cols) tile[ty + k][tx] = __ldg(in + (r0 + ty + k) * cols + c);
+            for (int e = t; e < kTT * kTT; e += kTThreads) {
+                const int i = e / kTT, j = e % kTT;
+                if (r0 + i < rows && c0 + j < cols) tile[i][j] = in[(r0 + i) * cols + c0 + j];
+            }
             __syncthreads();
-#pragma unroll
-            for (int k = 0; k < kTile; k += kRowsPerPass)
-                if (c0 + ty + k < cols && r0 + tx < rows) out[(c0 + ty + k) * rows + r0 + tx] = tile[tx][ty + k];
+            for (int e = t; e < kTT * kTT; e += kTThreads) {
+                const int j = e / kTT, i = e % kTT;
+                if (c0 + j < cols && r0 + i < rows) out[(c0 + j) * rows + r0 + i] = tile[i][j];
+            }
         }
         __syncthreads();
     }
@@ -44,13 +72,12 @@ transpose_kernel(const T *__restrict__ in, int64_t rows, int64_t cols, T *__rest
 
 template <typename T>
 static fs_status transpose_t(const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st) {
-    const int64_t tiles_r = ceil_div(rows, kTile), tiles_c = ceil_div(cols, kTile);
+    const int64_t tiles_r = ceil_div(rows, kTT), tiles_c = ceil_div(cols, kTT);
     const int64_t ntiles = tiles_r * tiles_c;
     if (ntiles == 0) return FS_OK;
-    const int64_t cap = resident_blocks((const void *)transpose_kernel<T>, kTile * kRowsPerPass) * 4;
+    const int64_t cap = resident_blocks((const void *)transpose_kernel<T>, kTThreads) * 8;
     const int64_t grid = ntiles < cap ? ntiles : cap;
-    transpose_kernel<T><<<(unsigned)grid, dim3(kTile, kRowsPerPass), 0, st>>>(
-        (const T *)in, rows, cols, (T *)out, tiles_c, ntiles);
+    transpose_kernel<T><<<(unsigned)grid, kTThreads, 0, st>>>((const T *)in, rows, cols, (T *)out, tiles_c, ntiles);
     return launch_status();
 }
 
