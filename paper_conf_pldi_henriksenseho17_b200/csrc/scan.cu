@@ -180,6 +180,20 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
     __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_val[NW];
     __shared__ int s_lb_min[NW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    // offset in its segment of this lane's first element of row q: one 64-bit modulo per
+    // tile, then steps of 32*VEC elements (rows of a lane's tile are 32*VEC apart)
+    const int64_t seg_step = SEG ? ((int64_t)32 * VEC) % L : 0;
+    int64_t seg_r0 = 0, seg_q0 = -1;
+    auto seg_off = [&](int64_t p0, int q) -> int64_t {
+        if (q == 0 || seg_q0 < 0) {
+            seg_r0 = p0 % L;
+        } else {
+            seg_r0 += seg_step;
+            if (seg_r0 >= L) seg_r0 -= L;
+        }
+        seg_q0 = q;
+        return seg_r0;
+    };
 
     if (threadIdx.x == 0) {
         if (TMA) {
@@ -252,7 +266,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
 #pragma unroll
                 for (int k = 0; k < VEC; ++k) xs[TMA ? 0 : q][k] = x[k];
             }
-            int64_t r = SEG ? (p0 % L) : 0;
+            int64_t r = SEG ? seg_off(p0, q) : 0;
             S run = SO::id();
 #pragma unroll
             for (int k = 0; k < VEC; ++k) {
@@ -363,7 +377,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
                 for (int k = 0; k < VEC; ++k) x[k] = xs[TMA ? 0 : q][k];
             }
             S run = SO::comb(base, pre[q]);
-            int64_t r = SEG ? (p0 % L) : 0;
+            int64_t r = SEG ? seg_off(p0, q) : 0;
             T y[VEC];
             int64_t yi[VEC];
 #pragma unroll
@@ -405,242 +419,6 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
     }
 }
 
-// ---------------------------------------------------------------- TMA tile scan
-// One tile at a time per CTA, several CTAs per SM:
-//   claim the next tile id (atomic counter: every predecessor is owned by a
-//   running CTA) -> TMA bulk load of the tile into shared memory -> local scan
-//   and publish the tile aggregate -> decoupled look-back over RB_WIN
-//   predecessors per step with the whole CTA (one status word per thread),
-//   "helping forward": when the window holds an inclusive prefix, every
-//   predecessor that only had an aggregate gets its inclusive prefix published
-//   too, so the next tiles find one a single step back -> write the tile.
-// A tile's aggregate is published one load + local scan after it was claimed,
-// so the look-back of the next tile rarely spins; the other CTAs on the SM
-// overlap this CTA's round trips.  (Claiming tiles ahead of processing made
-// successors spin on not-yet-published aggregates: measured slower.)
-template <int OP, typename T, bool SEG, int R>
-__global__ void __launch_bounds__(kScanThreads, 4)
-scan_tile_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
-                 int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
-                 TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
-    using O = Op<OP, T>;
-    using SO = SOp<O, SEG>;
-    using S = typename SO::S;
-    constexpr int VEC = 16 / sizeof(T), NW = kScanThreads / 32;
-    constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
-    constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
-    constexpr int WIN = kScanThreads;
-    extern __shared__ __align__(128) unsigned char sbuf[];
-    __shared__ uint64_t bar;
-    __shared__ int64_t s_tile;
-    __shared__ S s_wtot[NW], s_wex[NW], s_agg, s_ex, s_lb_tot[NW];
-    __shared__ int s_lb_min[NW];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    unsigned par = 0u;
-    if (threadIdx.x == 0) {
-        mbar_init(&bar, 1);
-        fence_mbar_init();
-    }
-    for (;;) {
-        FS_PROF_T(t1);
-        if (threadIdx.x == 0) {
-            const int64_t t = (int64_t)atomicAdd(counter, 1u);
-            s_tile = t;
-            if (t < ntiles && (t + 1) * TILE <= n) {
-                fence_proxy_async();
-                mbar_expect_tx(&bar, TILE_BYTES);
-                tma_load_1d(sbuf, in + t * TILE, TILE_BYTES, &bar);
-            }
-        }
-        __syncthreads();
-        const int64_t tile = s_tile;
-        if (tile >= ntiles) break;
-        FS_PROF_ADD(1, t1);
-        FS_PROF_T(t2);
-        const bool full = (tile + 1) * TILE <= n;
-        if (full) {
-            mbar_wait(&bar, par);
-            par ^= 1u;
-        }
-        FS_PROF_ADD(2, t2);
-        FS_PROF_T(t3);
-        const int64_t wbase = tile * TILE + (int64_t)warp * 32 * R * VEC;
-        auto load_row = [&](int q, T (&x)[VEC]) {
-            const int64_t p0 = wbase + ((int64_t)q * 32 + lane) * VEC;
-            if (full) {
-                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(sbuf + (((warp * R + q) * 32 + lane) << 4));
-#pragma unroll
-                for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
-            } else {
-#pragma unroll
-                for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
-            }
-            return p0;
-        };
-        auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
-            S e;
-            if (p0 + k < n) {
-                e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
-                e.f = SEG ? (r == 0) : 0;
-            } else {
-                e = SO::id();
-            }
-            if (SEG) {
-                ++r;
-                if (r == L) r = 0;
-            }
-            return e;
-        };
-        // local scan: per-row exclusive prefixes within the warp
-        S pre[R];
-        S carry_w = SO::id();
-#pragma unroll
-        for (int q = 0; q < R; ++q) {
-            T x[VEC];
-            const int64_t p0 = load_row(q, x);
-            int64_t r = SEG ? (p0 % L) : 0;
-            S run = SO::id();
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) run = SO::comb(run, lifted(x, p0, k, r));
-            S a = run;
-#pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const S o = SO::up(a, off);
-                if (lane >= off) a = SO::comb(o, a);
-            }
-            S ex = SO::up(a, 1);
-            if (lane == 0) ex = SO::id();
-            pre[q] = SO::comb(carry_w, ex);
-            carry_w = SO::comb(carry_w, SO::bcast(a, 31));
-        }
-        if (lane == 0) s_wtot[warp] = carry_w;
-        __syncthreads();
-        if (warp == 0) {
-            S a = lane < NW ? s_wtot[lane] : SO::id();
-#pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const S o = SO::up(a, off);
-                if (lane >= off) a = SO::comb(o, a);
-            }
-            S wex = SO::up(a, 1);
-            if (lane == 0) wex = SO::id();
-            if (lane < NW) s_wex[lane] = wex;
-            const S agg = SO::bcast(a, NW - 1);
-            if (lane == 0) {
-                s_agg = agg;
-                if (tile == 0) {
-                    S c0 = SO::id();
-                    if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-                    ts.publish(0, SO::comb(c0, agg), kStIncl);
-                } else {
-                    ts.publish(tile, agg, kStAgg);
-                }
-            }
-        }
-        __syncthreads();
-        FS_PROF_ADD(3, t3);
-        FS_PROF_T(t4);
-        // decoupled look-back
-        S exc = SO::id();
-        if (tile == 0) {
-            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-        } else {
-            int64_t j = tile - 1;
-            for (int step = 0;; ++step) {
-                const int64_t idx = j - threadIdx.x;
-                const bool mine = idx >= 0;
-                S v = SO::id();
-                unsigned st = kStIncl;
-                if (mine) {
-                    FS_PROF_T(t6);
-                    do {
-                        st = ts.poll(idx, v);
-#ifdef FS_SCAN_PROFILE
-                        if (threadIdx.x == 0 && st == 0) atomicAdd(&fs_scan_prof[7], 1ull);
-#endif
-                    } while (st == 0);
-                    FS_PROF_ADD(6, t6);
-                }
-                const unsigned m = __ballot_sync(0xffffffffu, mine && st == kStIncl);
-                if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
-                __syncthreads();
-#ifdef FS_SCAN_PROFILE
-                if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[8], 1ull);
-#endif
-                int kk = 1 << 20;
-#pragma unroll
-                for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
-                if ((int)threadIdx.x > kk || !mine) v = SO::id();
-                // suffix scan toward lower thread ids (higher ids are further left)
-                S a = v;
-#pragma unroll
-                for (int off = 1; off < 32; off <<= 1) {
-                    const S o = SO::down(a, off);
-                    if (lane + off < 32) a = SO::comb(o, a);
-                }
-                if (lane == 0) s_lb_tot[warp] = a;
-                __syncthreads();
-                S left = SO::id();
-#pragma unroll
-                for (int q = NW - 1; q > warp; --q) left = SO::comb(left, s_lb_tot[q]);
-                S P = SO::id();
-#pragma unroll
-                for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_tot[q]);
-                if (step == 0 && kk < (1 << 20) && mine && (int)threadIdx.x < kk && st == kStAgg)
-                    ts.publish(idx, SO::comb(left, a), kStIncl);  // help forward
-                exc = SO::comb(P, exc);
-                __syncthreads();
-                if (kk < (1 << 20) || exc.f) break;
-                j -= WIN;
-            }
-            if (threadIdx.x == 0) ts.publish(tile, SO::comb(exc, s_agg), kStIncl);
-        }
-        if (threadIdx.x == 0) s_ex = exc;
-        __syncthreads();
-        FS_PROF_ADD(4, t4);
-        FS_PROF_T(t5);
-        // write the tile
-        const S base = SO::comb(s_ex, s_wex[warp]);
-#pragma unroll
-        for (int q = 0; q < R; ++q) {
-            T x[VEC];
-            const int64_t p0 = load_row(q, x);
-            S run = SO::comb(base, pre[q]);
-            int64_t r = SEG ? (p0 % L) : 0;
-            T y[VEC];
-            int64_t yi[VEC];
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) {
-                run = SO::comb(run, lifted(x, p0, k, r));
-                y[k] = O::val(run.v);
-                yi[k] = O::idx(run.v);
-            }
-            if (p0 + VEC <= n) {
-                Vec16<T> w;
-#pragma unroll
-                for (int k = 0; k < VEC; ++k) w.e[k] = y[k];
-                int4 wv;
-                memcpy(&wv, &w, 16);
-                *reinterpret_cast<int4 *>(out + p0) = wv;
-            } else {
-#pragma unroll
-                for (int k = 0; k < VEC; ++k)
-                    if (p0 + k < n) out[p0 + k] = y[k];
-            }
-            if (OP == kArgmin) {
-#pragma unroll
-                for (int k = 0; k < VEC; ++k)
-                    if (p0 + k < n) out_idx[p0 + k] = yi[k];
-            }
-        }
-        __syncthreads();  // smem tile and s_tile reuse
-        FS_PROF_ADD(5, t5);
-#ifdef FS_SCAN_PROFILE
-        if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[0], 1ull);
-#endif
-    }
-}
-
 // ---------------------------------------------------------------- deferred look-back scan
 // Aggregates never wait; look-backs are deferred.  Iteration i of a CTA:
 //   A. claim tile t_i, TMA it from HBM, reduce it and publish its aggregate
@@ -670,6 +448,20 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
     __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_tot[NW];
     __shared__ int s_lb_min[NW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    // offset in its segment of this lane's first element of row q: one 64-bit modulo per
+    // tile, then steps of 32*VEC elements (rows of a lane's tile are 32*VEC apart)
+    const int64_t seg_step = SEG ? ((int64_t)32 * VEC) % L : 0;
+    int64_t seg_r0 = 0, seg_q0 = -1;
+    auto seg_off = [&](int64_t p0, int q) -> int64_t {
+        if (q == 0 || seg_q0 < 0) {
+            seg_r0 = p0 % L;
+        } else {
+            seg_r0 += seg_step;
+            if (seg_r0 >= L) seg_r0 -= L;
+        }
+        seg_q0 = q;
+        return seg_r0;
+    };
     unsigned par = 0u;
     auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
     auto issue = [&](int b, int64_t t) {
@@ -717,7 +509,7 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
         for (int q = 0; q < R; ++q) {
             T x[VEC];
             const int64_t p0 = load_row(b, t, q, x);
-            int64_t r = SEG ? (p0 % L) : 0;
+            int64_t r = SEG ? seg_off(p0, q) : 0;
             S run = SO::id();
 #pragma unroll
             for (int k = 0; k < VEC; ++k) run = SO::comb(run, lifted(x, p0, k, r));
@@ -746,6 +538,49 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
         const S agg = SO::bcast(a, NW - 1);
         __syncthreads();
         return agg;
+    };
+    // Aggregate of a tile for its look-back record, without scanning it: every table
+    // operator is commutative, so lanes fold their elements in any order and the CTA
+    // reduces; for the segmented operator only the elements at or after the tile's last
+    // segment start contribute, and that start is known in closed form (regular segments).
+    __shared__ typename O::V s_red[NW];
+    auto tile_aggregate = [&](int b, int64_t t) {
+        if (full_tile(t)) {
+            mbar_wait(&bars[b], (par >> b) & 1u);
+            par ^= 1u << b;
+        }
+        const int64_t t0 = t * TILE, t1 = (t + 1) * TILE < n ? (t + 1) * TILE : n;
+        int64_t keep = t0;
+        int flag = 0;
+        if (SEG) {
+            const int64_t last_start = ((t1 - 1) / L) * L;
+            flag = last_start >= t0;
+            keep = flag ? last_start : t0;
+        }
+        typename O::V acc = O::id();
+#pragma unroll
+        for (int q = 0; q < R; ++q) {
+            T x[VEC];
+            const int64_t p0 = load_row(b, t, q, x);
+            int64_t r = SEG ? seg_off(p0, q) : 0;
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) {
+                const int64_t pk = p0 + k;
+                if (pk < t1 && pk >= keep) acc = O::comb(acc, O::lift(x[k], SEG ? r : ibase + pk));
+                if (SEG) {
+                    ++r;
+                    if (r == L) r = 0;
+                }
+            }
+        }
+        acc = group_reduce<O>(acc);
+        if (lane == 0) s_red[warp] = acc;
+        __syncthreads();
+        typename O::V tot = O::id();
+#pragma unroll
+        for (int q = 0; q < NW; ++q) tot = O::comb(tot, s_red[q]);
+        __syncthreads();
+        return S{tot, flag};
     };
     auto carry_in = [&]() {
         S c0 = SO::id();
@@ -781,17 +616,22 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
             if (!more) break;
         }
         const int bA = (int)(i & 1), bC = 2 + (int)(i & 1);
+        FS_PROF_T(pa);
         // A. aggregate of the new tile
         if (ti < ntiles) {
-            const S agg = local_scan(bA, ti, pre);
+            const S agg = tile_aggregate(bA, ti);
             if (threadIdx.x == 0) {
                 if (ti == 0) ts.publish(0, SO::comb(carry_in(), agg), kStIncl);
                 else ts.publish(ti, agg, kStAgg);
             }
         }
+        FS_PROF_ADD(1, pa);
+        FS_PROF_T(pc);
         // C. scan + write the tile claimed D iterations ago
         if (told >= 0 && told < ntiles) {
             const S agg = local_scan(bC, told, pre);
+            FS_PROF_ADD(2, pc);
+            FS_PROF_T(pl);
             S exc = SO::id();
             if (told == 0) {
                 exc = carry_in();
@@ -839,13 +679,15 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
             }
             if (threadIdx.x == 0) s_ex = exc;
             __syncthreads();
+            FS_PROF_ADD(3, pl);
+            FS_PROF_T(pw);
             const S base = SO::comb(s_ex, s_wex[warp]);
 #pragma unroll
             for (int q = 0; q < R; ++q) {
                 T x[VEC];
                 const int64_t p0 = load_row(bC, told, q, x);
                 S run = SO::comb(base, pre[q]);
-                int64_t r = SEG ? (p0 % L) : 0;
+                int64_t r = SEG ? seg_off(p0, q) : 0;
                 T y[VEC];
                 int64_t yi[VEC];
 #pragma unroll
@@ -872,8 +714,12 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
                         if (p0 + k < n) out_idx[p0 + k] = yi[k];
                 }
             }
+            FS_PROF_ADD(4, pw);
         }
         __syncthreads();
+#ifdef FS_SCAN_PROFILE
+        if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[0], 1ull);
+#endif
     }
 }
 

@@ -4,6 +4,7 @@
 //        -Iinclude -Ipaper_conf_pldi_henriksenseho17_b200/csrc tools/scan_prof.cu \
 //        paper_conf_pldi_henriksenseho17_b200/csrc/{scan,api,redomap,colreduce,seg_reduce,stream_red,transpose}.cu -o scan_prof
 #include <cstdio>
+#include <cstdlib>
 #include <cuda_runtime.h>
 #include "futseg.h"
 extern "C" void fs_scan_prof_ptr(void **p);
@@ -17,19 +18,23 @@ int main() {
     fs_mapdesc m = {FS_MAP_ID, 0, 0, 0};
     size_t wb; fs_scanomap_workspace(op, n, &wb);
     cudaMalloc(&ws, wb); cudaMemset(ws, 0, wb);
-    for (int i = 0; i < 3; ++i) fs_scanomap(op, m, x, nullptr, n, y, nullptr, nullptr, nullptr, ws, wb, nullptr);
+    const int64_t L = getenv("SEGLEN") ? atoll(getenv("SEGLEN")) : 0;
+    auto run = [&]() {
+        return L ? fs_seg_scan(op, x, n / L, L, FS_ROW_MAJOR, y, nullptr, ws, wb, nullptr)
+                 : fs_scanomap(op, m, x, nullptr, n, y, nullptr, nullptr, nullptr, ws, wb, nullptr);
+    };
+    for (int i = 0; i < 3; ++i) run();
     cudaDeviceSynchronize();
     unsigned long long z[16] = {0};
     void *sym = nullptr; fs_scan_prof_ptr(&sym); cudaMemset(sym, 0, sizeof(z));
     cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
     cudaEventRecord(a);
-    int st = fs_scanomap(op, m, x, nullptr, n, y, nullptr, nullptr, nullptr, ws, wb, nullptr);
+    int st = run();
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
     cudaMemcpy(z, sym, sizeof(z), cudaMemcpyDeviceToHost);
     printf("status %d (%s) time %.3f ms  iterations %llu\n", st, cudaGetErrorString(cudaGetLastError()), ms, z[0]);
-    const char *names[] = {"iters", "claim+sync", "tma_wait", "phaseA+publish", "lookback", "phaseC+sync",
-                           "lb: t0 poll cycles", "lb: t0 respins", "lb: steps"};
-    for (int i = 1; i < 9; ++i) printf("%-20s %10.1f cycles/iter\n", names[i], (double)z[i] / (double)z[0]);
+    const char *names[] = {"iters", "A: wait+scan+publish", "C: wait+local scan", "C: look-back", "C: write"};
+    for (int i = 1; i < 5; ++i) printf("%-20s %10.1f cycles/iter\n", names[i], (double)z[i] / (double)z[0]);
     return 0;
 }
