@@ -286,10 +286,18 @@ def main():
         print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch N>1 with torch.distributed.run",
               file=sys.stderr)
         sys.exit(2)
+    # FUTSEG_BENCH_DEVICE0=1 + FUTSEG_BENCH_BACKEND=gloo: every rank on cuda:0 over gloo -- a
+    # functional check of the N > 1 path on a one-GPU box (not a performance number)
+    if os.environ.get("FUTSEG_BENCH_DEVICE0") == "1":
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        tdist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("FUTSEG_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            tdist.init_process_group("nccl", device_id=dev)
+        else:
+            tdist.init_process_group(backend)
     import paper_conf_pldi_henriksenseho17_b200 as fs
 
     W = build_workload(fs, dev, rank, world, args.quick)

@@ -186,7 +186,9 @@ template <int OP, typename T> struct RedomapNN {
         const bool vect = (((uintptr_t)lat ^ (uintptr_t)lng) & 15) == 0;
         const void *k = vect ? (const void *)redomap_nn_kernel<OP, kRedThreads, kRedU, true>
                              : (const void *)redomap_nn_kernel<OP, kRedThreads, kRedU, false>;
-        const int64_t per_cta = (int64_t)kRedThreads * kRedU * 4;
+        // the distance map costs ~40 instructions per record: spread small inputs (NN's
+        // 855,280 records) over the whole machine, one 4-record vector per thread minimum
+        const int64_t per_cta = (int64_t)kRedThreads * 4;
         int64_t grid = ceil_div(n, per_cta);
         grid = grid < 1 ? 1 : grid;
         const int64_t cap = resident_blocks(k, kRedThreads);

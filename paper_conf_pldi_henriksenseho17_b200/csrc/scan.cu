@@ -178,7 +178,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
     __shared__ uint64_t bars[2];
     __shared__ int64_t s_tile[2];
     __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_val[NW];
-    __shared__ int s_lb_min[NW];
+    __shared__ __align__(16) int s_lb_min[NW];  // aligned: the min over it is read with 16-byte loads
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     // offset in its segment of this lane's first element of row q: one 64-bit modulo per
     // tile, then steps of 32*VEC elements (rows of a lane's tile are 32*VEC apart)
@@ -446,7 +446,7 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
     __shared__ uint64_t bars[4];
     __shared__ int64_t s_ring[RING];
     __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_tot[NW];
-    __shared__ int s_lb_min[NW];
+    __shared__ __align__(16) int s_lb_min[NW];  // aligned: the min over it is read with 16-byte loads
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     // offset in its segment of this lane's first element of row q: one 64-bit modulo per
     // tile, then steps of 32*VEC elements (rows of a lane's tile are 32*VEC apart)

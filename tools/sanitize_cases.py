@@ -1,0 +1,46 @@
+"""Small invocations of every libfutseg primitive for compute-sanitizer (tools/sanitize.sh)."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import workloads  # noqa: E402
+import paper_conf_pldi_henriksenseho17_b200 as fs  # noqa: E402
+
+
+def cu(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+x = cu(workloads.mixed(300_001, 1, np.float32))
+xi = cu(workloads.mixed(300_001, 2, np.int64))
+for op in ("add", "min", "argmin"):
+    fs.redomap(x, op)
+    fs.redomap(xi, op)
+    fs.scanomap(x, op)
+    fs.scanomap(xi[1:], op)
+lat, lng, q = workloads.c2_nn(base=20_000, reps=2)
+fs.redomap(cu(lat), "argmin", map="nn_dist", lng=cu(lng), query=q)
+fs.scanomap(cu(lat), "min", map="nn_dist", lng=cu(lng), query=q)
+fs.redomap(cu(workloads.mixed((5000, 34), 3, np.float32)), "vadd")
+for nseg, L in ((10_000, 1), (7_001, 3), (4096, 32), (1000, 33), (300, 1000), (20, 10_000), (2, 150_000)):
+    m = x[: nseg * L]
+    for reg in (-1, 0, 1, 2, 3):
+        fs.force_seg_regime(reg)
+        fs.seg_reduce(m, nseg, L, "add")
+        fs.seg_reduce(m, nseg, L, "argmin")
+    fs.force_seg_regime(-1)
+    fs.seg_reduce(m, nseg, L, "max", layout="col")
+    fs.seg_scan(m, nseg, L, "add")
+    fs.seg_scan(m, nseg, L, "argmin", layout="col")
+pts, mem = workloads.c3_kmeans(n=30_000, d=34, k=5)
+fs.stream_red(cu(pts), cu(mem), 5)
+pts, mem = workloads.c3_kmeans(n=30_000, d=34, k=32)
+fs.stream_red(cu(pts), cu(mem), 32)
+fs.stream_red(cu(workloads.mixed((3000, 100), 4, np.float32)), cu(workloads.ints(3000, 5, 0, 70)), 70)
+fs.transpose_2d(cu(workloads.mixed((333, 517), 6, np.float32)))
+fs.transpose_2d(cu(workloads.mixed((256, 128), 7, np.int64)))
+torch.cuda.synchronize()
+print("sanitize cases done")
