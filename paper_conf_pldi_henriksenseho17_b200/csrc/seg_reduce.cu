@@ -107,7 +107,7 @@ __device__ __forceinline__ void small_segs(const Vec16<T> &e, int64_t v, T *out,
 }
 
 template <int OP, typename T, int NT, int U>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT, 4)
 seg_vec_kernel(const T *__restrict__ x, int64_t nseg, int L, int G, T *out, int64_t *out_idx) {
     using O = Op<OP, T>;
     using V = typename O::V;
@@ -131,27 +131,40 @@ seg_vec_kernel(const T *__restrict__ x, int64_t nseg, int L, int G, T *out, int6
     if (iters > 0) load_batch(0, r);
     for (int64_t it0 = 0; it0 < iters; it0 += U) {
         if (it0 + U < iters) load_batch(it0 + U, rn);
+        if (L <= VEC) {
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int64_t v = gid0 + (it0 + u) * stride;
-            const bool live = it0 + u < iters;  // warp-uniform
-            const bool ok = live && v < nvec;
-            const Vec16<T> e = as_vec<T>(r[u]);
-            if (L <= VEC) {
-                if (ok) {
+            for (int u = 0; u < U; ++u) {
+                const int64_t v = gid0 + (it0 + u) * stride;
+                if (it0 + u < iters && v < nvec) {
+                    const Vec16<T> e = as_vec<T>(r[u]);
                     if (L == 1) small_segs<O, T, 1>(e, v, out, out_idx);
                     else if (L == 2) small_segs<O, T, 2>(e, v, out, out_idx);
                     else small_segs<O, T, (VEC >= 4 ? 4 : VEC)>(e, v, out, out_idx);
                 }
-            } else {
-                V a = O::id();
-                if (ok) {
+            }
+        } else {
+            // in-lane fold of each vector, then the xor-shuffle steps with the U vectors
+            // interleaved (independent chains: the shuffle latency overlaps)
+            V a[U];
 #pragma unroll
-                    for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], (int64_t)lg * VEC + k);
+            for (int u = 0; u < U; ++u) {
+                const int64_t v = gid0 + (it0 + u) * stride;
+                a[u] = O::id();
+                if (it0 + u < iters && v < nvec) {
+                    const Vec16<T> e = as_vec<T>(r[u]);
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) a[u] = O::fold(a[u], e.e[k], (int64_t)lg * VEC + k);
                 }
-                if (live)
-                    for (int m = G >> 1; m >= 1; m >>= 1) a = O::comb(a, shfl_xor(a, m));
-                if (ok && lg == 0) store_out<O>(out, out_idx, v / G, a);
+            }
+#pragma unroll 1
+            for (int m = G >> 1; m >= 1; m >>= 1) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) a[u] = O::comb(a[u], shfl_xor(a[u], m));
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t v = gid0 + (it0 + u) * stride;
+                if (it0 + u < iters && v < nvec && lg == 0) store_out<O>(out, out_idx, v / G, a[u]);
             }
         }
 #pragma unroll
