@@ -181,7 +181,8 @@ fs_status fs_seg_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, in
     if (!bytes) return FS_ERR_NULL;
     FS_TRY(check_op(op, false));
     if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return FS_ERR_SIZE;
-    if (layout == FS_ROW_MAJOR) *bytes = seg_reduce_ws(op.op, op.dtype, nseg, seglen);
+    if (layout == FS_ROW_MAJOR || (layout == FS_COL_MAJOR && (nseg <= 1 || seglen <= 1)))
+        *bytes = seg_reduce_ws(op.op, op.dtype, nseg, seglen);
     else if (layout == FS_COL_MAJOR) *bytes = colreduce_ws(op.op, op.dtype, seglen, nseg);
     else return FS_ERR_UNSUPPORTED;
     return FS_OK;
@@ -191,7 +192,8 @@ fs_status fs_seg_scan_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, int3
     if (!bytes) return FS_ERR_NULL;
     FS_TRY(check_op(op, false));
     if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return FS_ERR_SIZE;
-    if (layout == FS_ROW_MAJOR) *bytes = scan_ws(op.op, op.dtype, nseg * seglen);
+    if (layout == FS_ROW_MAJOR || (layout == FS_COL_MAJOR && (nseg <= 1 || seglen <= 1)))
+        *bytes = scan_ws(op.op, op.dtype, nseg * seglen);
     else if (layout == FS_COL_MAJOR) *bytes = colscan_ws(op.op, op.dtype, seglen, nseg);
     else return FS_ERR_UNSUPPORTED;
     return FS_OK;
@@ -326,7 +328,9 @@ fs_status fs_seg_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t segl
     int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
     if (nseg == 0) return FS_OK;
     if (seglen == 0) return fill_neutral_run(op.op, op.dtype, nseg, out, oi, S(stream));
-    if (layout == FS_COL_MAJOR) return colreduce_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
+    // with one segment, or segments of one element, both layouts are the same bytes
+    if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1)
+        return colreduce_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
     return seg_reduce_run(op.op, op.dtype, in, nseg, seglen, out, oi, ws, S(stream));
 }
 
@@ -338,8 +342,9 @@ fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen
     FS_TRY(check_ws(ws, ws_bytes, need));
     int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
     if (nseg * seglen == 0) return FS_OK;
-    if (layout == FS_COL_MAJOR) return colscan_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
-    const fs_mapdesc id = {FS_MAP_ID, 0.f, 0.f};
+    if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1)
+        return colscan_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
+    const fs_mapdesc id = {FS_MAP_ID, 0.f, 0.f, 0};
     return scan_run(op.op, op.dtype, id, in, nullptr, nseg * seglen, seglen, out, oi, nullptr, nullptr, ws,
                     S(stream));
 }
@@ -374,7 +379,7 @@ int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t 
     if (check_op(op, false) != FS_OK || nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return -1;
     if (layout != FS_ROW_MAJOR && layout != FS_COL_MAJOR) return -1;
     if (nseg == 0 || seglen == 0) return 6;
-    if (layout == FS_COL_MAJOR) return 4;
+    if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1) return 4;
     if (prim_is_scan) return 5;
     return seg_reduce_regime(op.op, op.dtype, nseg, seglen);
 }

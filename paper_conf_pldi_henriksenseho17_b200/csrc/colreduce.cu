@@ -136,6 +136,11 @@ static ColPlan col_plan(int dt, int64_t m, int64_t w, bool aligned, int op, int6
     const int64_t wv = ceil_div(w, p.vec);
     p.CG = (int)(wv < kColThreads ? wv : kColThreads);
     if (p.CG < 1) p.CG = 1;
+    // narrower column tiles when columns are few: enough tiles that each needs at most
+    // ~64 row splits, so the last CTA of a tile folds few partial rows (a single CTA
+    // folding hundreds of partial rows serialised the wide, short case)
+    const int64_t want_tiles = resident / 64 > 1 ? resident / 64 : 1;
+    while (p.CG > 32 && ceil_div(wv, p.CG) < want_tiles) p.CG /= 2;
     p.tiles = ceil_div(wv, p.CG);
     const int RB = kColThreads / p.CG;
     // row splits: fill the machine, keep >= 16 rows per thread-row, and keep the

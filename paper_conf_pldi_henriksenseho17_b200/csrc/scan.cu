@@ -823,7 +823,27 @@ colscan_partial_kernel(const T *__restrict__ x, int64_t m, int64_t w, int64_t WV
 #pragma unroll
     for (int k = 0; k < VEC; ++k) acc[k] = O::id();
     const T *base = x + cv * VEC;
-    for (int64_t r = r0; r < r1; ++r) {
+    constexpr int UR = 8;  // rows in flight per thread
+    int64_t r = r0;
+    for (; r + UR <= r1; r += UR) {
+        Vec16<T> e[UR];
+        T s1[UR];
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+            if (VEC > 1) e[u] = as_vec<T>(ldg16(base + (r + u) * w));
+            else s1[u] = __ldg(base + (r + u) * w);
+        }
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+            if (VEC > 1) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], e[u].e[k], r + u);
+            } else {
+                acc[0] = O::fold(acc[0], s1[u], r + u);
+            }
+        }
+    }
+    for (; r < r1; ++r) {
         if (VEC > 1) {
             const Vec16<T> e = as_vec<T>(*reinterpret_cast<const int4 *>(base + r * w));
 #pragma unroll
@@ -862,6 +882,31 @@ __global__ void colscan_carry_kernel(typename Op<OP, T>::V *partials, int64_t w,
     }
 }
 
+// exclusive scan over the Y row blocks of ONE column per CTA (few columns, many
+// row blocks): each thread folds a contiguous run of row blocks, the CTA scans the
+// per-thread totals, then each thread rewrites its run with the carries
+template <int OP, typename T>
+__global__ void __launch_bounds__(256) colscan_carry_block_kernel(typename Op<OP, T>::V *partials, int64_t w, int64_t Y) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    __shared__ V s_tot[256];
+    const int64_t c = blockIdx.x;
+    const int t = threadIdx.x;
+    const int64_t chunk = (Y + 255) / 256;
+    const int64_t y0 = t * chunk, y1 = y0 + chunk < Y ? y0 + chunk : Y;
+    V a = O::id();
+    for (int64_t y = y0; y < y1; ++y) a = O::comb(a, partials[y * w + c]);
+    s_tot[t] = a;
+    __syncthreads();
+    V run = O::id();
+    for (int q = 0; q < t; ++q) run = O::comb(run, s_tot[q]);  // exclusive prefix of the runs
+    for (int64_t y = y0; y < y1; ++y) {
+        const V p = partials[y * w + c];
+        partials[y * w + c] = run;
+        run = O::comb(run, p);
+    }
+}
+
 template <int OP, typename T, int VEC, bool CARRY>
 __global__ void __launch_bounds__(kColScanThreads)
 colscan_kernel(const T *__restrict__ x, int64_t m, int64_t w, int64_t WV, int64_t Y, int64_t rpu,
@@ -877,7 +922,38 @@ colscan_kernel(const T *__restrict__ x, int64_t m, int64_t w, int64_t WV, int64_
     for (int k = 0; k < VEC; ++k) acc[k] = CARRY ? carries[y * w + cv * VEC + k] : O::id();
     const T *base = x + cv * VEC;
     T *obase = out + cv * VEC;
-    for (int64_t r = r0; r < r1; ++r) {
+    constexpr int UR = 8;  // rows loaded ahead per thread
+    int64_t r = r0;
+    for (; r + UR <= r1; r += UR) {
+        Vec16<T> e[UR];
+        T s1[UR];
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+            if (VEC > 1) e[u] = as_vec<T>(ldg16(base + (r + u) * w));
+            else s1[u] = __ldg(base + (r + u) * w);
+        }
+#pragma unroll
+        for (int u = 0; u < UR; ++u) {
+            const int64_t rr = r + u;
+            if (VEC > 1) {
+                Vec16<T> o;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) {
+                    acc[k] = O::comb(acc[k], O::lift(e[u].e[k], rr));
+                    o.e[k] = O::val(acc[k]);
+                    if (OP == kArgmin) out_idx[rr * w + cv * VEC + k] = O::idx(acc[k]);
+                }
+                int4 ov;
+                memcpy(&ov, &o, 16);
+                *reinterpret_cast<int4 *>(obase + rr * w) = ov;
+            } else {
+                acc[0] = O::comb(acc[0], O::lift(s1[u], rr));
+                obase[rr * w] = O::val(acc[0]);
+                if (OP == kArgmin) out_idx[rr * w + cv] = O::idx(acc[0]);
+            }
+        }
+    }
+    for (; r < r1; ++r) {
         if (VEC > 1) {
             const Vec16<T> e = as_vec<T>(*reinterpret_cast<const int4 *>(base + r * w));
             Vec16<T> o;
@@ -931,9 +1007,13 @@ template <int OP, typename T> struct ColScanRun {
             return launch_status();
         }
         colscan_partial_kernel<OP, T, VEC><<<grid, kColScanThreads, 0, st>>>(x, m, w, p.WV, p.Y, p.rpu, parts);
-        int64_t g2 = ceil_div(w, 128);
-        g2 = g2 > 4096 ? 4096 : g2;
-        colscan_carry_kernel<OP, T><<<(unsigned)g2, 128, 0, st>>>(parts, w, p.Y);
+        if (p.Y >= 256) {  // few columns, many row blocks: one CTA per column
+            colscan_carry_block_kernel<OP, T><<<(unsigned)w, 256, 0, st>>>(parts, w, p.Y);
+        } else {
+            int64_t g2 = ceil_div(w, 128);
+            g2 = g2 > 4096 ? 4096 : g2;
+            colscan_carry_kernel<OP, T><<<(unsigned)g2, 128, 0, st>>>(parts, w, p.Y);
+        }
         colscan_kernel<OP, T, VEC, true><<<grid, kColScanThreads, 0, st>>>(x, m, w, p.WV, p.Y, p.rpu, parts, out,
                                                                            out_idx);
         return launch_status(3);
