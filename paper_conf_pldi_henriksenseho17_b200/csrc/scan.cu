@@ -129,7 +129,10 @@ __device__ __forceinline__ float nn_dist_s(float lat, float lng, float q0, float
 #ifndef FS_SCAN_R
 #define FS_SCAN_R 4
 #endif
-constexpr int kScanThreads = 256;
+#ifndef FS_SCAN_NT
+#define FS_SCAN_NT 128  // swept on B200 (64/128/256 threads x R = 2/4/8): 128 x 4 fastest
+#endif
+constexpr int kScanThreads = FS_SCAN_NT;
 constexpr unsigned kStAgg = 1, kStIncl = 2;
 
 // -DFS_SCAN_PROFILE: thread 0 of every CTA accumulates clock64 cycles per phase of
@@ -162,7 +165,7 @@ template <int OP, typename T> struct ScanShape {
 // runs the decoupled look-back (warp 0) and writes the tile.  With TMA the next
 // tile's HBM read overlaps this tile's scan, look-back and store.
 template <int OP, typename T, bool NN, bool SEG, bool TMA>
-__global__ void __launch_bounds__(kScanThreads, TMA ? 3 : 2)
+__global__ void __launch_bounds__(kScanThreads, (TMA ? 768 : 512) / kScanThreads)
 scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n, int64_t L, float q0, float q1,
             int64_t ibase, T *__restrict__ out, int64_t *__restrict__ out_idx, const T *carry,
             const int64_t *carry_idx, unsigned *counter, TileState<typename SOp<Op<OP, T>, SEG>::S,
@@ -430,7 +433,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
 //      inclusive prefix (helping forward) and write it.
 // HBM traffic stays one read + one write per element; the second read hits L2.
 template <int OP, typename T, bool SEG, int R, int D>
-__global__ void __launch_bounds__(kScanThreads, 3)
+__global__ void __launch_bounds__(kScanThreads, 768 / kScanThreads)
 scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
                int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
                TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
