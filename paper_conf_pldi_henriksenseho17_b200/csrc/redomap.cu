@@ -11,6 +11,8 @@
 // -- the combine of sFold's chunk results (L259-260) without a second launch.
 // The fused map (identity or the Rodinia NN distance) is applied in registers:
 // the mapped array is never materialised (L1815-1817: fusion).
+#include <stdlib.h>
+
 #include "internal.cuh"
 
 namespace fs {

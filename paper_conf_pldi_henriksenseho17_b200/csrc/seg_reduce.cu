@@ -181,6 +181,63 @@ seg_vec_kernel(const T *__restrict__ x, int64_t nseg, int L, int G, T *out, int6
     }
 }
 
+// ---------------------------------------------------------------- KG0, wide lanes
+// Power-of-two L >= UPL*VEC: each lane folds UPL consecutive 16-byte vectors
+// (a 64-byte run) of one segment in registers, so a segment spans
+// G = L / (UPL*VEC) lanes and needs log2(G) xor shuffles instead of
+// log2(L/VEC).  A warp instruction reads 16 B per lane at a 64-B stride; the
+// L1-allocating loads let the four instructions of a run share their sectors.
+template <int OP, typename T, int NT, int U, int UPL>
+__global__ void __launch_bounds__(NT, 4)
+seg_vecw_kernel(const T *__restrict__ x, int64_t nseg, int L, int G, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    constexpr int RUN = UPL * VEC;  // elements per lane run
+    const int lane = threadIdx.x & 31;
+    const int64_t nrun = nseg * (int64_t)L / RUN;
+    const int64_t stride = (int64_t)gridDim.x * NT;
+    const int lg = lane & (G - 1);
+    const int64_t gid0 = (int64_t)blockIdx.x * NT + threadIdx.x;
+    const int64_t iters = (nrun + stride - 1) / stride;
+    for (int64_t it0 = 0; it0 < iters; it0 += U) {
+        int4 r[U][UPL];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            if (it0 + u < iters && v < nrun) {
+                const int4 *p = reinterpret_cast<const int4 *>(x + v * RUN);
+#pragma unroll
+                for (int j = 0; j < UPL; ++j) r[u][j] = __ldg(p + j);
+            }
+        }
+        V a[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            a[u] = O::id();
+            if (it0 + u < iters && v < nrun) {
+#pragma unroll
+                for (int j = 0; j < UPL; ++j) {
+                    const Vec16<T> e = as_vec<T>(r[u][j]);
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) a[u] = O::fold(a[u], e.e[k], (int64_t)lg * RUN + j * VEC + k);
+                }
+            }
+        }
+#pragma unroll 1
+        for (int m = G >> 1; m >= 1; m >>= 1) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) a[u] = O::comb(a[u], shfl_xor(a[u], m));
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            if (it0 + u < iters && v < nrun && lg == 0) store_out<O>(out, out_idx, v / G, a[u]);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- KG2
 template <int OP, typename T, int NT, int U>
 __global__ void __launch_bounds__(NT)
@@ -314,7 +371,7 @@ int seg_reduce_regime(int op, int dt, int64_t nseg, int64_t L) {
         return forced;
     }
     const int64_t vec = 16 / (int64_t)dtype_size(dt);
-    if (L <= 64 || ((L & (L - 1)) == 0 && L <= 32 * vec)) return 0;  // KG1 (KG0 when L is a power of two)
+    if (L <= 64 || ((L & (L - 1)) == 0 && L <= 4 * 32 * vec / 2)) return 0;  // KG1 (KG0 when L is a power of two)
     if (L <= kWarpMaxL) return 1;
     const int64_t resident = (int64_t)sm_count() * 8;
     return nseg >= 2 * resident ? 2 : 3;
@@ -348,6 +405,18 @@ template <int OP, typename T> struct SegRun {
         const T *x = (const T *)in;
         constexpr int VEC = 16 / sizeof(T);
         const bool pow2 = (L & (L - 1)) == 0;
+        constexpr int UPL = 4;
+        if (regime == 0 && pow2 && L >= UPL * VEC && L <= 32 * UPL * VEC && ((uintptr_t)x & 15) == 0) {
+            const int G = (int)(L / (UPL * VEC));
+            const void *k = (const void *)seg_vecw_kernel<OP, T, kSegThreads, 2, UPL>;
+            const int64_t nrun = nseg * L / (UPL * VEC);
+            int64_t grid = ceil_div(nrun > 0 ? nrun : 1, (int64_t)kSegThreads * 2);
+            const int64_t cap = resident_blocks(k, kSegThreads);
+            grid = grid < cap ? grid : cap;
+            seg_vecw_kernel<OP, T, kSegThreads, 2, UPL><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, G,
+                                                                                            (T *)out, out_idx);
+            return launch_status();
+        }
         if (regime == 0 && pow2 && L <= 32 * VEC && ((uintptr_t)x & 15) == 0) {
             const int G = L > VEC ? (int)(L / VEC) : 1;
             const void *k = (const void *)seg_vec_kernel<OP, T, kSegThreads, 4>;
