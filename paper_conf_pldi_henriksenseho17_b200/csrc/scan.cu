@@ -650,6 +650,9 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
                             st = ts.poll(idx, v);
                         } while (st == 0);
                     }
+#ifdef FS_SCAN_PROFILE
+                    if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[5], 1ull);
+#endif
                     const unsigned m = __ballot_sync(0xffffffffu, mine && st == kStIncl);
                     if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
                     __syncthreads();

@@ -34,7 +34,8 @@ int main() {
     float ms; cudaEventElapsedTime(&ms, a, b);
     cudaMemcpy(z, sym, sizeof(z), cudaMemcpyDeviceToHost);
     printf("status %d (%s) time %.3f ms  iterations %llu\n", st, cudaGetErrorString(cudaGetLastError()), ms, z[0]);
-    const char *names[] = {"iters", "A: wait+scan+publish", "C: wait+local scan", "C: look-back", "C: write"};
-    for (int i = 1; i < 5; ++i) printf("%-20s %10.1f cycles/iter\n", names[i], (double)z[i] / (double)z[0]);
+    const char *names[] = {"iters", "A: wait+reduce+publish", "C: wait+local scan", "C: look-back", "C: write",
+                           "look-back steps"};
+    for (int i = 1; i < 6; ++i) printf("%-20s %10.1f cycles/iter\n", names[i], (double)z[i] / (double)z[0]);
     return 0;
 }
