@@ -124,6 +124,50 @@ colreduce_kernel(const T *__restrict__ x, int64_t m, int64_t w, int CG, int64_t 
     if (t == 0) atomicExch(tickets + blockIdx.x, 0u);
 }
 
+// Many columns, few rows (one split): each thread owns one vector column and walks
+// all m rows (U loads in flight), writing its outputs directly; a grid-stride loop
+// over vector columns keeps the grid at the resident size instead of one CTA per
+// 1024-column tile.
+template <int OP, typename T, int NT, int VEC, int U>
+__global__ void __launch_bounds__(NT)
+colreduce_direct_kernel(const T *__restrict__ x, int64_t m, int64_t w, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    const int64_t WV = w / VEC;
+    for (int64_t cv = (int64_t)blockIdx.x * NT + threadIdx.x; cv < WV; cv += (int64_t)gridDim.x * NT) {
+        V acc[VEC];
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) acc[k] = O::id();
+        const T *base = x + cv * VEC;
+        int64_t r = 0;
+        for (; r + U <= m; r += U) {
+            Vec16<T> e[U];
+            T s1[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (VEC > 1) e[u] = as_vec<T>(ldg16(base + (r + u) * w));
+                else s1[u] = __ldg(base + (r + u) * w);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], VEC > 1 ? e[u].e[k] : s1[u], r + u);
+            }
+        }
+        for (; r < m; ++r) {
+            if (VEC > 1) {
+                const Vec16<T> e = as_vec<T>(ldg16(base + r * w));
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], e.e[k], r);
+            } else {
+                acc[0] = O::fold(acc[0], __ldg(base + r * w), r);
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) store_out<O>(out, out_idx, cv * VEC + k, acc[k]);
+    }
+}
+
 struct ColPlan {
     int vec, CG;
     int64_t tiles, Y, rows_per_split;
@@ -166,6 +210,17 @@ template <int OP, typename T> struct ColRun {
         const bool aligned = ((uintptr_t)in & 15) == 0;
         const int64_t resident = (int64_t)sm_count() * 8;
         const ColPlan p = col_plan(sizeof(T) == 8 ? FS_I64 : FS_I32, m, w, aligned, OP, resident);
+        const int64_t WV = p.vec > 1 ? w / p.vec : w;
+        if (p.Y == 1 && WV >= resident * kColThreads) {  // many columns, few rows
+            const int64_t grid = ceil_div(WV, kColThreads) < resident * 2 ? ceil_div(WV, kColThreads) : resident * 2;
+            if (p.vec > 1)
+                colreduce_direct_kernel<OP, T, kColThreads, VV, 4><<<(unsigned)grid, kColThreads, 0, st>>>(
+                    (const T *)in, m, w, (T *)out, out_idx);
+            else
+                colreduce_direct_kernel<OP, T, kColThreads, 1, 4><<<(unsigned)grid, kColThreads, 0, st>>>(
+                    (const T *)in, m, w, (T *)out, out_idx);
+            return launch_status();
+        }
         char *wsb = (char *)ws;
         V *parts = (V *)(wsb + kWsHeader);
         unsigned *tickets = (unsigned *)(wsb + kWsTickets);  // p.Y > 1 implies p.tiles <= kWsMaxTickets
