@@ -244,6 +244,23 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
     }
 }
 
+// 1-D bulk copy shared -> global (SASS UBLKCP), tracked by bulk async-groups of the
+// issuing thread: commit after issuing, wait_group_read<N> before the source smem
+// is overwritten (all but the N most recent groups have finished READING smem),
+// wait_group<0> before exit (writes performed).
+__device__ __forceinline__ void tma_store_1d(void *dst, const void *src, unsigned bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+template <int N> __device__ __forceinline__ void bulk_wait() {
+    asm volatile("cp.async.bulk.wait_group %0;" ::"n"(N) : "memory");
+}
+
 // ------------------------------------------------------------------ workspace layout
 // [0, 256)          : control words
 //     u32 ticket   @ 0     (single-counter kernels; reset by the last CTA)

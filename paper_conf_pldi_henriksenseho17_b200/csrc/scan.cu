@@ -730,6 +730,715 @@ scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
 }
 
 // ws body: [0,256) tile counter | status words (8 B per tile) | aggs | incls
+// ---------------------------------------------------------------- thread-contiguous TMA scan
+// The default path for 16-byte aligned inputs and outputs.  Every tile moves
+// HBM -> shared memory by one TMA bulk load and shared memory -> HBM by one TMA
+// bulk store; threads never touch global memory for a full tile.  Thread t owns
+// the R contiguous 16-byte vectors t*R .. t*R+R-1 of the tile (R odd: the eight
+// threads of a 16-byte shared-memory wavefront hit eight distinct bank groups),
+// so a tile costs one sequential fold per element, one warp scan and one block
+// scan of per-thread totals, and one (+) per element to apply the prefix, which
+// is written back in place and stored by TMA.  The ST-stage ring keeps ST-2
+// tiles of loads in flight per CTA while a tile is scanned and one is drained
+// by its bulk store; two CTAs per SM overlap one CTA's look-back wait with the
+// other's work.  Tiles are claimed in order from an atomic counter (forward
+// progress); the look-back window is the whole CTA.  For the segmented
+// operator a tile whose aggregate carries a segment start publishes it as its
+// inclusive prefix at once ((e, agg) = agg when agg.f, footnote 5's operator),
+// and a tile that starts a segment never looks back.
+#ifndef FS_SCANT_NT
+#define FS_SCANT_NT 256
+#endif
+#ifndef FS_SCANT_R
+#define FS_SCANT_R 3
+#endif
+#ifndef FS_SCANT_ST
+#define FS_SCANT_ST 5
+#endif
+#ifndef FS_SCANT_DYN
+#define FS_SCANT_DYN 0
+#endif
+#ifndef FS_SCANT_AHEAD
+#define FS_SCANT_AHEAD 1
+#endif
+#ifndef FS_SCANT_MINB
+#define FS_SCANT_MINB 3
+#endif
+constexpr int kScanTThreads = FS_SCANT_NT;
+template <int OP, typename T> struct ScanTShape {
+    static constexpr bool PACK = OP != kArgmin && sizeof(T) == 4;
+    static constexpr int R = PACK ? FS_SCANT_R : 3;
+    static_assert(R % 2 == 1, "R must be odd (bank-conflict-free thread-contiguous vectors)");
+    static constexpr int ST = FS_SCANT_ST;
+    static_assert(ST >= 3, "ring needs >= 3 stages (aggregates run one tile ahead of the scan)");
+    static constexpr int VEC = 16 / sizeof(T);
+    static constexpr int E = R * VEC;  // elements per thread per tile
+    static constexpr int64_t TILE = (int64_t)kScanTThreads * E;
+    static constexpr unsigned TILE_BYTES = kScanTThreads * R * 16;
+};
+
+template <int OP, typename T, bool SEG>
+__global__ void __launch_bounds__(kScanTThreads, FS_SCANT_MINB)
+scan_tc_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+               int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
+               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanTShape<OP, T>::PACK> ts, int64_t ntiles) {
+    using O = Op<OP, T>;
+    using SO = SOp<O, SEG>;
+    using S = typename SO::S;
+    using Sh = ScanTShape<OP, T>;
+    constexpr int VEC = Sh::VEC, R = Sh::R, E = Sh::E, ST = Sh::ST, NW = kScanTThreads / 32;
+    constexpr int64_t TILE = Sh::TILE;
+    constexpr unsigned TB = Sh::TILE_BYTES;
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    __shared__ uint64_t bars[ST];
+    __shared__ int64_t s_tile[ST];
+    __shared__ S s_wtot[NW], s_lb_val[NW];
+    __shared__ int s_lb_min[NW];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
+    // static round-robin tiles: iteration `it` of this CTA scans tile blockIdx.x + it * gridDim.x
+    // (grid <= resident CTAs, so every tile is owned by a running CTA that visits its
+    // tiles in increasing order: forward progress)
+    auto tile_of = [&](int it) {
+        return FS_SCANT_DYN ? s_tile[it % ST] : (int64_t)blockIdx.x + (int64_t)it * gridDim.x;
+    };
+    auto issue = [&](int it) {  // thread 0 only
+        const int s = it % ST;
+        if (FS_SCANT_DYN) s_tile[s] = (int64_t)atomicAdd(counter, 1u);
+        const int64_t t = tile_of(it);
+        if (t < ntiles && full_tile(t)) {
+            fence_proxy_async();
+            mbar_expect_tx(&bars[s], TB);
+            tma_load_1d(sbuf + s * TB, in + t * TILE, TB, &bars[s]);
+        }
+    };
+
+    // per-tile state carried from phase A (aggregate, one iteration ahead) to phase C
+    struct Pre {
+        S tex, wex, agg;
+    };
+    auto load_x = [&](int s, int64_t tile, bool full, int64_t e0, T (&x)[E]) {
+        if (full) {
+            const unsigned char *sv = sbuf + s * TB + threadIdx.x * (R * 16);
+#pragma unroll
+            for (int j = 0; j < R; ++j) {
+                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(sv + j * 16);
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) x[j * VEC + k] = a.e[k];
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < E; ++i) x[i] = e0 + i < n ? in[e0 + i] : T(0);
+        }
+    };
+    auto lifted = [&](const T (&x)[E], bool full, int64_t e0, int i, int64_t &r) {
+        S e;
+        if (full || e0 + i < n) {
+            e.v = O::lift(x[i], SEG ? r : ibase + e0 + i);
+            e.f = SEG ? (r == 0) : 0;
+        } else {
+            e = SO::id();
+        }
+        if (SEG) {
+            ++r;
+            if (r == L) r = 0;
+        }
+        return e;
+    };
+    // phase A of iteration `it`: wait for the tile, fold, warp + block scan of thread
+    // totals, publish the aggregate (or the inclusive prefix when it needs no look-back)
+    auto phase_a = [&](int it, Pre &p) {
+        const int s = it % ST;
+        const int64_t tile = tile_of(it);
+        const bool full = full_tile(tile);
+        const int64_t e0 = tile * TILE + (int64_t)threadIdx.x * E;
+        if (full) mbar_wait(&bars[s], (unsigned)(it / ST) & 1u);
+        T x[E];
+        load_x(s, tile, full, e0, x);
+        S tot = SO::id();
+        int64_t r = SEG ? e0 % L : 0;
+#pragma unroll
+        for (int i = 0; i < E; ++i) tot = SO::comb(tot, lifted(x, full, e0, i, r));
+        S a = tot;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const S o = SO::up(a, off);
+            if (lane >= off) a = SO::comb(o, a);
+        }
+        p.tex = SO::up(a, 1);
+        if (lane == 0) p.tex = SO::id();
+        if (lane == 31) s_wtot[warp] = a;
+        __syncthreads();
+        S b = lane < NW ? s_wtot[lane] : SO::id();
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const S o = SO::up(b, off);
+            if (lane >= off) b = SO::comb(o, b);
+        }
+        S bex = SO::up(b, 1);
+        if (lane == 0) bex = SO::id();
+        p.wex = SO::bcast(bex, warp);
+        p.agg = SO::bcast(b, NW - 1);
+        if (threadIdx.x == 0) {
+            if (tile == 0) {
+                S c0 = SO::id();
+                if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+                ts.publish(0, SO::comb(c0, p.agg), kStIncl);
+            } else {
+                // a flagged aggregate is already the inclusive prefix
+                ts.publish(tile, p.agg, (SEG && p.agg.f) ? kStIncl : kStAgg);
+            }
+        }
+    };
+
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int s = 0; s < ST; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+#pragma unroll
+        for (int q = 0; q < ST - 1; ++q) issue(q);
+    }
+    __syncthreads();
+    Pre cur, nxt;
+    if (FS_SCANT_AHEAD && tile_of(0) < ntiles) phase_a(0, cur);
+    for (int it = 0;; ++it) {
+        const int s = it % ST;
+        const int64_t tile = tile_of(it);
+        if (tile >= ntiles) break;
+        const bool full = full_tile(tile);
+        const int64_t e0 = tile * TILE + (int64_t)threadIdx.x * E;
+        // aggregate of the next tile first: it never waits on anything but its own data
+        if (!FS_SCANT_AHEAD) phase_a(it, cur);
+        else if (tile_of(it + 1) < ntiles) phase_a(it + 1, nxt);
+        // ---- look-back for this tile (its predecessors published at least an iteration ago)
+        S exc = SO::id();
+        if (tile == 0) {
+            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+        } else if (!(SEG && (tile * TILE) % L == 0)) {
+            int64_t j = tile - 1;
+            while (true) {
+                const int64_t idx = j - threadIdx.x;
+                S v = SO::id();
+                unsigned st = kStIncl;
+                if (idx >= 0) {
+                    do {
+                        st = ts.poll(idx, v);
+                    } while (st == 0);
+                }
+                const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
+                if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 30;
+                __syncthreads();
+                int kk = 1 << 30;
+#pragma unroll
+                for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
+                if ((int)threadIdx.x > kk || idx < 0) v = SO::id();
+                S w = v;
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const S o = SO::down(w, off);
+                    if (lane + off < 32) w = SO::comb(o, w);
+                }
+                if (lane == 0) s_lb_val[warp] = w;
+                __syncthreads();
+                S P = SO::id(), left = SO::id();
+#pragma unroll
+                for (int q = NW - 1; q >= 0; --q) {
+                    if (q > warp) left = SO::comb(left, s_lb_val[q]);
+                    P = SO::comb(P, s_lb_val[q]);
+                }
+                // help forward: a predecessor found as an aggregate between this tile and the
+                // nearest inclusive prefix gets its inclusive prefix published now
+                if (kk < (1 << 30) && idx >= 0 && (int)threadIdx.x < kk && st == kStAgg)
+                    ts.publish(idx, SO::comb(left, w), kStIncl);
+                exc = SO::comb(P, exc);
+                __syncthreads();  // s_lb_* reuse
+                if (kk < (1 << 30) || exc.f || j < kScanTThreads) break;
+                j -= kScanTThreads;
+            }
+            if (threadIdx.x == 0 && !(SEG && cur.agg.f)) ts.publish(tile, SO::comb(exc, cur.agg), kStIncl);
+        }
+        // ---- phase C: apply the prefix; full tiles go back in place and out by one bulk store
+        {
+            T x[E];
+            load_x(s, tile, full, e0, x);
+            S run = SO::comb(exc, SO::comb(cur.wex, cur.tex));
+            int64_t r = SEG ? e0 % L : 0;
+            T y[E];
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                run = SO::comb(run, lifted(x, full, e0, i, r));
+                y[i] = O::val(run.v);
+                if (OP == kArgmin && (full || e0 + i < n)) out_idx[e0 + i] = O::idx(run.v);
+            }
+            if (full) {
+                unsigned char *sv = sbuf + s * TB + threadIdx.x * (R * 16);
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    Vec16<T> w;
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) w.e[k] = y[j * VEC + k];
+                    *reinterpret_cast<Vec16<T> *>(sv + j * 16) = w;
+                }
+                fence_proxy_async();  // generic-proxy smem writes -> visible to the bulk store
+            } else {
+#pragma unroll
+                for (int i = 0; i < E; ++i)
+                    if (e0 + i < n) out[e0 + i] = y[i];
+            }
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (full) tma_store_1d(out + tile * TILE, sbuf + s * TB, TB);
+            bulk_commit();
+            bulk_wait_read<1>();  // the store of stage (it-1)%ST has read its smem
+            issue(it + ST - 1);
+        }
+        if (FS_SCANT_AHEAD) cur = nxt;
+    }
+    if (threadIdx.x == 0) bulk_wait<0>();
+}
+
+// ---------------------------------------------------------------- warp-specialised slab scan
+// The default path for 16-byte aligned inputs and outputs.  One CTA per SM.  The
+// array is cut into tiles of TILE_BYTES and the tiles into slabs of `tps`
+// consecutive tiles; CTA b owns slabs b, b+G, b+2G, ... (a "round" is G consecutive
+// slabs).  Three warp roles run concurrently in every CTA:
+//   A (4 warps)  REDUCE each slab as it streams from HBM through an STA-stage TMA
+//                ring: the slab's look-back record is a commutative masked reduction
+//                (for the segmented operator only elements at or after the slab's last
+//                segment start count -- a closed form for regular segments), published
+//                as soon as the slab has been read.
+//   C (8 warps)  per slab: one decoupled look-back over the records of the preceding
+//                slabs (window 256 >= G, one L2 round trip per slab), then scan the slab
+//                tile by tile with a running carry from an STC-stage ring that re-reads
+//                it from L2 (group A read it a moment ago), thread-contiguous R (odd)
+//                vectors per thread (bank-conflict free), results written back in place.
+//   P (1 warp)   the producer: issues every TMA load of both rings and the TMA bulk
+//                store of every scanned tile, driven by mbarriers (A/C "slot consumed",
+//                C "tile written back"); keeps group A at most DA slabs ahead of C so
+//                the slabs between the two passes stay in L2 (G*(DA+1) slabs).
+// HBM traffic is one read and one write per element.  This is F5 (L1071-1074) in
+// B200 form: A computes the chunk aggregates, C the chunk scans with the carried
+// prefix a, and the look-back composes the carries.
+#ifndef FS_SCANW_R
+#define FS_SCANW_R 7
+#endif
+#ifndef FS_SCANW_STA
+#define FS_SCANW_STA 4
+#endif
+#ifndef FS_SCANW_STC
+#define FS_SCANW_STC 3
+#endif
+#ifndef FS_SCANW_DA
+#define FS_SCANW_DA 2
+#endif
+#ifndef FS_SCANW_TPS
+#define FS_SCANW_TPS 4
+#endif
+#ifndef FS_SCANW_NC
+#define FS_SCANW_NC 256
+#endif
+constexpr int kScanWA = 128, kScanWC = FS_SCANW_NC, kScanWThreads = kScanWA + kScanWC + 32;
+template <int OP, typename T> struct ScanWShape {
+    static constexpr bool PACK = OP != kArgmin && sizeof(T) == 4;
+    static constexpr int R = FS_SCANW_R;  // C: 16-byte vectors per thread per tile
+    static_assert(R % 2 == 1, "R must be odd (bank-conflict-free thread-contiguous vectors)");
+    static constexpr int VEC = 16 / sizeof(T);
+    static constexpr int E = R * VEC;
+    static constexpr int64_t TILE = (int64_t)kScanWC * E;
+    static constexpr unsigned TILE_BYTES = kScanWC * R * 16;
+    static constexpr int RA = kScanWC * R / kScanWA;  // A: vectors per thread per tile
+    static_assert(kScanWC * R % kScanWA == 0, "A threads split a tile evenly");
+    static constexpr int STA = FS_SCANW_STA, STC = FS_SCANW_STC;
+    static constexpr unsigned SMEM = (STA + STC) * TILE_BYTES;
+};
+
+__device__ __forceinline__ void named_bar(int id, int count) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+__device__ __forceinline__ bool mbar_test(uint64_t *bar, unsigned parity) {
+    uint32_t done;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return done != 0;
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void tma_load_1d_hint(void *dst, const void *src, unsigned bytes, uint64_t *bar,
+                                                 uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], "
+        "%4;" ::"r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ void tma_store_1d_hint(void *dst, const void *src, unsigned bytes, uint64_t pol) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(dst),
+                 "r"(smem_u32(src)), "r"(bytes), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_wait_read_n(int n) {  // all but the n most recent groups have read
+    if (n <= 0) bulk_wait_read<0>();
+    else if (n == 1) bulk_wait_read<1>();
+    else if (n == 2) bulk_wait_read<2>();
+    else bulk_wait_read<3>();
+}
+
+template <int OP, typename T, bool SEG>
+__global__ void __launch_bounds__(kScanWThreads, 1)
+scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+               int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx,
+               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanWShape<OP, T>::PACK> ts, int64_t ntiles, int tps) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    using SO = SOp<O, SEG>;
+    using S = typename SO::S;
+    using Sh = ScanWShape<OP, T>;
+    constexpr int VEC = Sh::VEC, R = Sh::R, E = Sh::E, RA = Sh::RA, STA = Sh::STA, STC = Sh::STC;
+    constexpr int NWA = kScanWA / 32, NWC = kScanWC / 32;
+    constexpr int64_t TILE = Sh::TILE;
+    constexpr unsigned TB = Sh::TILE_BYTES;
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    unsigned char *ringA = sbuf, *ringC = sbuf + STA * TB;
+    __shared__ uint64_t fullA[STA], emptyA[STA], fullC[STC], doneC[STC];
+    __shared__ volatile int s_c_slab;  // slab (local index) group C is working on
+    __shared__ V s_redA[NWA];
+    __shared__ S s_wtot[2][NWC], s_lb_val[NWC];
+    __shared__ int s_lb_min[NWC];
+    const int G = gridDim.x, b = blockIdx.x;
+    const int64_t nslabs = (ntiles + tps - 1) / tps;
+    const int my_slabs = (int)((nslabs - b + G - 1) / G);
+    // tile sequence of this CTA: j -> (local slab j / tps, tile j % tps of it)
+    auto slab_of = [&](int m) { return (int64_t)b + (int64_t)m * G; };
+    auto tile_at = [&](int j) { return slab_of(j / tps) * tps + j % tps; };
+    const int my_tiles = my_slabs == 0 ? 0 : (int)((my_slabs - 1) * (int64_t)tps +
+                                                   (min((int64_t)tps, ntiles - slab_of(my_slabs - 1) * tps)));
+    auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        for (int s = 0; s < STA; ++s) {
+            mbar_init(&fullA[s], 1);
+            mbar_init(&emptyA[s], kScanWA);
+        }
+        for (int s = 0; s < STC; ++s) {
+            mbar_init(&fullC[s], 1);
+            mbar_init(&doneC[s], kScanWC);
+        }
+        fence_mbar_init();
+        s_c_slab = 0;
+    }
+    __syncthreads();
+
+    if (tid >= kScanWA + kScanWC) {
+        // ================================================================ P: producer
+        if (tid != kScanWA + kScanWC) return;
+        const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
+        int a_iss = 0, a_rel = 0, c_iss = 0, c_st = 0;
+        while (c_st < my_tiles) {
+            // A: a slot is released when all of group A has consumed its tile
+            while (a_rel < a_iss && mbar_test(&emptyA[a_rel % STA], (unsigned)(a_rel / STA) & 1u)) ++a_rel;
+            // A: issue while a slot is free and A stays within DA slabs of C
+            while (a_iss < my_tiles && a_iss < a_rel + STA && a_iss / tps - FS_SCANW_DA <= s_c_slab) {
+                const int64_t t = tile_at(a_iss);
+                if (full_tile(t)) {
+                    const int s = a_iss % STA;
+                    mbar_expect_tx(&fullA[s], TB);
+                    tma_load_1d_hint(ringA + s * TB, in + t * TILE, TB, &fullA[s], keep);
+                }
+                ++a_iss;
+            }
+            // C: store every tile group C has written back (in order)
+            while (c_st < c_iss && mbar_test(&doneC[c_st % STC], (unsigned)(c_st / STC) & 1u)) {
+                const int64_t t = tile_at(c_st);
+                if (full_tile(t)) tma_store_1d_hint(out + t * TILE, ringC + (c_st % STC) * TB, TB, stream);
+                bulk_commit();
+                ++c_st;
+            }
+            // C: re-load (from L2) tiles group A has finished, into slots whose store has read them
+            while (c_iss < my_tiles && c_iss < a_rel && c_iss < c_st + STC) {
+                const int old = c_iss - STC;  // previous tile of this slot; its store is group `old`
+                if (old >= 0) bulk_wait_read_n(c_st - 1 - old);
+                const int64_t t = tile_at(c_iss);
+                if (full_tile(t)) {
+                    const int s = c_iss % STC;
+                    fence_proxy_async();
+                    mbar_expect_tx(&fullC[s], TB);
+                    tma_load_1d_hint(ringC + s * TB, in + t * TILE, TB, &fullC[s], stream);
+                }
+                ++c_iss;
+            }
+        }
+        bulk_wait<0>();
+        return;
+    }
+    if (tid < kScanWA) {
+        // ================================================================ A: slab records
+        const int lane = tid & 31, warp = tid >> 5;
+        int j = 0;
+        for (int m = 0; m < my_slabs; ++m) {
+            const int64_t slab = slab_of(m);
+            const int64_t s0 = slab * tps * TILE, s1 = min(n, (slab + 1) * tps * TILE);
+            // SEG: the record covers the slab's elements from its last segment start on (all
+            // of them when no segment starts in it); they lie in ONE segment starting at `base`
+            int64_t keep = s0, base = 0;
+            int flag = 0;
+            if (SEG) {
+                const int64_t last_start = ((s1 - 1) / L) * L;
+                flag = last_start >= s0;
+                keep = flag ? last_start : s0;
+                base = flag ? last_start : (s0 / L) * L;
+            }
+            V acc = O::id();
+            const int64_t t_end = min(ntiles, (slab + 1) * tps);
+            for (int64_t t = slab * tps; t < t_end; ++t, ++j) {
+                const int s = j % STA;
+                const bool full = full_tile(t);
+                const int64_t t0 = t * TILE, t1 = t0 + TILE;
+                if (full) mbar_wait(&fullA[s], (unsigned)(j / STA) & 1u);
+                if (SEG && t1 <= keep) {
+                    // entirely before the slab's last segment start: not part of the record
+                } else if (full && (!SEG || t0 >= keep)) {
+#pragma unroll
+                    for (int q = 0; q < RA; ++q) {
+                        const int vi = q * kScanWA + tid;
+                        const int64_t p0 = t0 + (int64_t)vi * VEC;
+                        const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(ringA + s * TB + vi * 16);
+#pragma unroll
+                        for (int k = 0; k < VEC; ++k)
+                            acc = O::comb(acc, O::lift(a.e[k], SEG ? p0 + k - base : ibase + p0 + k));
+                    }
+                } else {
+#pragma unroll
+                    for (int q = 0; q < RA; ++q) {
+                        const int vi = q * kScanWA + tid;
+                        const int64_t p0 = t0 + (int64_t)vi * VEC;
+                        T x[VEC];
+                        if (full) {
+                            const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(ringA + s * TB + vi * 16);
+#pragma unroll
+                            for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
+                        } else {
+#pragma unroll
+                            for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
+                        }
+#pragma unroll
+                        for (int k = 0; k < VEC; ++k) {
+                            const int64_t pk = p0 + k;
+                            if (pk < s1 && (!SEG || pk >= keep))
+                                acc = O::comb(acc, O::lift(x[k], SEG ? pk - base : ibase + pk));
+                        }
+                    }
+                }
+                mbar_arrive(&emptyA[s]);
+            }
+            acc = group_reduce<O>(acc);
+            if (lane == 0) s_redA[warp] = acc;
+            named_bar(1, kScanWA);
+            if (tid == 0) {
+                V tot = O::id();
+#pragma unroll
+                for (int q = 0; q < NWA; ++q) tot = O::comb(tot, s_redA[q]);
+                S agg{tot, flag};
+                if (slab == 0) {
+                    S c0 = SO::id();
+                    if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+                    ts.publish(0, SO::comb(c0, agg), kStIncl);
+                } else {
+                    // a flagged record is already the inclusive prefix
+                    ts.publish(slab, agg, (SEG && flag) ? kStIncl : kStAgg);
+                }
+            }
+            named_bar(1, kScanWA);  // s_redA reuse
+        }
+        return;
+    }
+    // ==================================================================== C: look-back + scan
+    const int ct = tid - kScanWA, lane = ct & 31, warp = ct >> 5;
+    int j = 0;
+    for (int m = 0; m < my_slabs; ++m) {
+        const int64_t slab = slab_of(m);
+        if (ct == 0) s_c_slab = m;
+        S exc = SO::id();
+        if (slab == 0) {
+            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
+        } else if (!(SEG && (slab * tps * TILE) % L == 0)) {
+            int64_t jj = slab - 1;
+            while (true) {
+                const int64_t idx = jj - ct;
+                S v = SO::id();
+                unsigned st = kStIncl;
+                if (idx >= 0) {
+                    do {
+                        st = ts.poll(idx, v);
+                    } while (st == 0);
+                }
+                const unsigned msk = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
+                if (lane == 0) s_lb_min[warp] = msk ? warp * 32 + __ffs(msk) - 1 : 1 << 30;
+                named_bar(2, kScanWC);
+                int kk = 1 << 30;
+#pragma unroll
+                for (int q = 0; q < NWC; ++q) kk = min(kk, s_lb_min[q]);
+                if (ct > kk || idx < 0) v = SO::id();
+                S w = v;
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    const S o = SO::down(w, off);
+                    if (lane + off < 32) w = SO::comb(o, w);
+                }
+                if (lane == 0) s_lb_val[warp] = w;
+                named_bar(2, kScanWC);
+                S P = SO::id(), left = SO::id();
+#pragma unroll
+                for (int q = NWC - 1; q >= 0; --q) {
+                    if (q > warp) left = SO::comb(left, s_lb_val[q]);
+                    P = SO::comb(P, s_lb_val[q]);
+                }
+                // help forward: records between here and the nearest inclusive prefix
+                if (kk < (1 << 30) && idx >= 0 && ct < kk && st == kStAgg) ts.publish(idx, SO::comb(left, w), kStIncl);
+                exc = SO::comb(P, exc);
+                named_bar(2, kScanWC);  // s_lb_* reuse
+                if (kk < (1 << 30) || exc.f || jj < kScanWC) break;
+                jj -= kScanWC;
+            }
+        }
+        S run_c = exc;
+        const int64_t t_end = min(ntiles, (slab + 1) * tps);
+        // offset in its segment of this thread's first element: one division per slab
+        int64_t r0 = SEG ? (slab * tps * TILE + (int64_t)ct * E) % L : 0;
+        for (int64_t t = slab * tps; t < t_end; ++t, ++j) {
+            const int s = j % STC;
+            const bool full = full_tile(t);
+            const int64_t e0 = t * TILE + (int64_t)ct * E;
+            unsigned char *sv = ringC + s * TB + ct * (R * 16);
+            T x[E];
+            if (full) {
+                mbar_wait(&fullC[s], (unsigned)(j / STC) & 1u);
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(sv + r * 16);
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) x[r * VEC + k] = a.e[k];
+                }
+            } else {
+#pragma unroll
+                for (int i = 0; i < E; ++i) x[i] = e0 + i < n ? in[e0 + i] : T(0);
+            }
+            auto valid = [&](int i) { return full || e0 + i < n; };
+            // SEG with L >= E: at most one segment start among a thread's E elements, at i0
+            const bool one = SEG && L >= E;
+            const int i0 = !SEG ? E : (r0 == 0 ? 0 : (L - r0 < E ? (int)(L - r0) : E));
+            auto lifted = [&](int i, int64_t &r) {
+                S e;
+                if (valid(i)) {
+                    e.v = O::lift(x[i], SEG ? r : ibase + e0 + i);
+                    e.f = SEG ? (r == 0) : 0;
+                } else {
+                    e = SO::id();
+                }
+                if (SEG) {
+                    ++r;
+                    if (r == L) r = 0;
+                }
+                return e;
+            };
+            auto seg_idx = [&](int i) -> int64_t { return i < i0 ? r0 + i : i - i0; };  // one-start case
+            S tot = SO::id();
+            if (one) {
+                V acc = O::id();
+#pragma unroll
+                for (int i = 0; i < E; ++i)
+                    if (valid(i)) {
+                        const V e = O::lift(x[i], seg_idx(i));
+                        acc = i == i0 ? e : O::comb(acc, e);
+                    }
+                tot = S{acc, i0 < E};
+            } else {
+                int64_t r = r0;
+#pragma unroll
+                for (int i = 0; i < E; ++i) tot = SO::comb(tot, lifted(i, r));
+            }
+            S a = tot;
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {
+                const S o = SO::up(a, off);
+                if (lane >= off) a = SO::comb(o, a);
+            }
+            S tex = SO::up(a, 1);
+            if (lane == 0) tex = SO::id();
+            if (lane == 31) s_wtot[j & 1][warp] = a;
+            named_bar(2, kScanWC);
+            S bsc = lane < NWC ? s_wtot[j & 1][lane] : SO::id();
+#pragma unroll
+            for (int off = 1; off < NWC; off <<= 1) {
+                const S o = SO::up(bsc, off);
+                if (lane >= off) bsc = SO::comb(o, bsc);
+            }
+            S bex = SO::up(bsc, 1);
+            if (lane == 0) bex = SO::id();
+            const S wex = SO::bcast(bex, warp), tagg = SO::bcast(bsc, NWC - 1);
+            S run = SO::comb(run_c, SO::comb(wex, tex));
+            run_c = SO::comb(run_c, tagg);
+            T y[E];
+            if (one) {
+                V acc = run.v;
+#pragma unroll
+                for (int i = 0; i < E; ++i) {
+                    if (valid(i)) {
+                        const V e = O::lift(x[i], seg_idx(i));
+                        acc = i == i0 ? e : O::comb(acc, e);
+                    }
+                    y[i] = O::val(acc);
+                    if (OP == kArgmin && valid(i)) out_idx[e0 + i] = O::idx(acc);
+                }
+            } else {
+                int64_t r = r0;
+#pragma unroll
+                for (int i = 0; i < E; ++i) {
+                    run = SO::comb(run, lifted(i, r));
+                    y[i] = O::val(run.v);
+                    if (OP == kArgmin && valid(i)) out_idx[e0 + i] = O::idx(run.v);
+                }
+            }
+            if (SEG) {
+                r0 += TILE % L;
+                if (r0 >= L) r0 -= L;
+            }
+            if (full) {
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    Vec16<T> w;
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) w.e[k] = y[r * VEC + k];
+                    *reinterpret_cast<Vec16<T> *>(sv + r * 16) = w;
+                }
+                fence_proxy_async();  // written back -> visible to the producer's bulk store
+            } else {
+#pragma unroll
+                for (int i = 0; i < E; ++i)
+                    if (e0 + i < n) out[e0 + i] = y[i];
+            }
+            mbar_arrive(&doneC[s]);
+        }
+        // the slab's inclusive prefix (group A may already have published an equal one)
+        if (ct == 0) ts.publish(slab, run_c, kStIncl);
+    }
+    if (ct == 0) s_c_slab = 1 << 30;
+}
+
 static size_t scan_state_bytes(int64_t ntiles) { return align_up((size_t)ntiles * 8, 256); }
 
 template <int OP, typename T> struct ScanRun {
@@ -750,6 +1459,34 @@ template <int OP, typename T> struct ScanRun {
         }
         if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntiles), st) != cudaSuccess) return FS_ERR_CUDA;
         if constexpr (TMA && !NN) {
+#ifndef FS_SCAN_TC
+            {
+                using ShW = ScanWShape<OP, T>;
+                const int64_t ntw = ceil_div(n, ShW::TILE);
+                const int64_t G0 = sm_count();
+                int64_t tps = ntw / (G0 * 4);
+                tps = tps < 1 ? 1 : (tps > FS_SCANW_TPS ? FS_SCANW_TPS : tps);
+                const int64_t nslabs = ceil_div(ntw, tps);
+                const int64_t G = nslabs < G0 ? nslabs : G0;
+                auto kw = scan_ws_kernel<OP, T, SEG>;
+                cudaFuncSetAttribute((const void *)kw, cudaFuncAttributeMaxDynamicSharedMemorySize, ShW::SMEM);
+                kw<<<(unsigned)G, kScanWThreads, ShW::SMEM, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
+                                                                  (const T *)carry, carry_idx, ts, ntw, (int)tps);
+                return launch_status();
+            }
+#endif
+#ifndef FS_SCAN_DEFERRED
+            using ShB = ScanTShape<OP, T>;
+            const int64_t ntb = ceil_div(n, ShB::TILE);
+            auto kb = scan_tc_kernel<OP, T, SEG>;
+            const int smemb = ShB::ST * (int)ShB::TILE_BYTES;
+            cudaFuncSetAttribute((const void *)kb, cudaFuncAttributeMaxDynamicSharedMemorySize, smemb);
+            const int64_t capb = resident_blocks((const void *)kb, kScanTThreads, smemb);
+            const int64_t gridb = ntb < capb ? ntb : capb;
+            kb<<<(unsigned)gridb, kScanTThreads, smemb, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
+                                                               (const T *)carry, carry_idx, counter, ts, ntb);
+            return launch_status();
+#endif
             // same tile shape as the ws sizing (Sh::R rows of 16-byte vectors per thread)
             // deferred look-back, 4 buffers of half-size tiles (same tile grid as the ws sizing)
             // D = 3 iterations of deferral (swept 1..3 and R = 4/8 on B200: R4 D3 fastest)

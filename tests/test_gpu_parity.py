@@ -139,7 +139,7 @@ def test_combine(fs, op):
 # ------------------------------------------------------------------ scanomap
 @pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("op", OPS)
-@pytest.mark.parametrize("n,offset", [(1, 0), (5, 1), (4096, 0), (100_003, 0), (1_000_003, 2)])
+@pytest.mark.parametrize("n,offset", [(1, 0), (5, 1), (4096, 0), (100_003, 0), (1_000_003, 2), (5_000_011, 0)])
 def test_scanomap(fs, dt, op, n, offset):
     x = workloads.mixed(n, 200 + n, dt)
     got = fs.scanomap(cu(x, offset), op)
