@@ -267,8 +267,8 @@ def test_stream_red_c3_kdd_shape(fs, keys):
 
 
 @pytest.mark.parametrize("dt", DTYPES)
-@pytest.mark.parametrize("k,w", [(1, 1), (3, 7), (8, 32), (5, 33), (16, 64), (32, 34), (32, 64), (33, 10),
-                                 (100, 70), (7, 200), (300, 100), (2000, 40)])
+@pytest.mark.parametrize("k,w", [(1, 1), (3, 7), (8, 32), (5, 33), (16, 64), (32, 34), (32, 36), (32, 37),
+                                 (9, 35), (32, 64), (33, 10), (100, 70), (7, 200), (300, 100), (2000, 40)])
 def test_stream_red_shapes(fs, dt, k, w):
     n = 30_011
     vals = workloads.mixed((n, w), k * 100 + w, dt)
@@ -278,6 +278,39 @@ def test_stream_red_shapes(fs, dt, k, w):
     np.testing.assert_array_equal(host(counts), wc)
     absum = oracle.stream_red(np.abs(vals), mem, k)[0] if dt == np.float32 else None
     assert_reduced(sums, ws, "add", absum, f"stream_red k={k} w={w}")
+
+
+@pytest.mark.parametrize("k,w", [(32, 34), (5, 34), (32, 36), (8, 40)])
+def test_stream_red_skewed_staged(fs, k, w):
+    """TMA-staged path with skewed keys (90% in cluster 0): the cluster-owner lane of the
+    extra features walks up to a whole stage of rows; every chunk's ragged tail too."""
+    n = 200_003
+    pts, mem = workloads.c3_kmeans(n=n, d=w, k=k, keys="skewed", seed=11)
+    sums, counts = fs.stream_red(cu(pts), cu(mem), k)
+    ws, wc = oracle.stream_red(pts, mem, k)
+    np.testing.assert_array_equal(host(counts), wc)
+    assert_reduced(sums, ws, "add", ws, f"stream_red skewed k={k} w={w}")
+
+
+def test_stream_red_bad_key_staged(fs):
+    """An out-of-range key inside a TMA stage is skipped (trash row) and flagged; the
+    other rows of that stage still count."""
+    n = 100_000
+    vals = workloads.mixed((n, 34), 5, np.float32)
+    mem = workloads.ints(n, 6, 0, 32)
+    bad = [17, 40_000, 99_999]
+    fs.check_device_error()
+    mem_bad = mem.copy()
+    mem_bad[bad] = [32, -1, 1 << 30]
+    sums, counts = fs.stream_red(cu(vals), cu(mem_bad), 32)
+    with pytest.raises(fs.FutsegError, match="BOUNDS"):
+        fs.check_device_error()
+    keep = np.ones(n, bool)
+    keep[bad] = False
+    ws, wc = oracle.stream_red(vals[keep], mem[keep], 32)
+    np.testing.assert_array_equal(host(counts), wc)
+    absum, _ = oracle.stream_red(np.abs(vals[keep]), mem[keep], 32)
+    assert_reduced(sums, ws, "add", absum, "stream_red bad keys staged")
 
 
 def test_stream_red_small_and_empty(fs):
