@@ -59,8 +59,9 @@ def _L():
         lib.orc_seg_scan.argtypes = [I, I, P, L, L, I, P, P]
         lib.orc_stream_red.argtypes = [I, P, P, L, L, L, P, P]
         lib.orc_transpose.argtypes = [L, P, L, L, P]
+        lib.orc_nn_knn.argtypes = [P, P, L, ctypes.c_float, ctypes.c_float, L, P, P, P, P]
         for f in ("orc_reduce", "orc_scan", "orc_nn_dist", "orc_vreduce", "orc_seg_reduce",
-                  "orc_seg_scan", "orc_stream_red", "orc_transpose"):
+                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn"):
             getattr(lib, f).restype = I
         _lib = lib
     return _lib
@@ -111,6 +112,22 @@ def nn_dist(lat, lng, q0, q1):
     out = np.zeros(lat.size, np.float32)
     _check(_L().orc_nn_dist(_p(lat), _p(lng), lat.size, float(q0), float(q1), _p(out)), "nn_dist")
     return out
+
+
+def nn_knn(lat, lng, q, kk):
+    """NEXT-2: Rodinia NN's kk nearest neighbours as kk rounds of the argmin reduce over
+    the distance map, each round excluding its winner (L1653-1655, reading R16).
+    Returns (dist[kk] f32, idx[kk] int64); rounds beyond n give (+inf, -1)."""
+    lat = np.ascontiguousarray(lat, np.float32)
+    lng = np.ascontiguousarray(lng, np.float32)
+    n = lat.size
+    dist = np.zeros(kk, np.float32)
+    idx = np.zeros(kk, np.int64)
+    ds = np.zeros(max(n, 1), np.float32)
+    ch = np.zeros(max(n, 1), np.uint8)
+    _check(_L().orc_nn_knn(_p(lat), _p(lng), n, float(q[0]), float(q[1]), kk, _p(dist), _p(idx), _p(ds), _p(ch)),
+           "nn_knn")
+    return dist, idx
 
 
 def redomap(x, op="add", map="id", lng=None, q=(0.0, 0.0)):

@@ -256,3 +256,35 @@ int orc_transpose(int64_t esize, const void *in, int64_t rows, int64_t cols, voi
             memcpy(dst + (j * rows + i) * esize, src + (i * cols + j) * esize, (size_t)esize);
     return 0;
 }
+
+/* NEXT-2, Rodinia NN's "100 reduce operations for finding the nearest
+ * neighbors" (L1653-1655; reading R16): kk rounds of the argmin reduce of
+ * R3 over the distance map of R5, each round excluding the record it found.
+ *   round r: (out_dist[r], out_idx[r]) = argmin over not-yet-chosen i of
+ *            (dist[i], i), first occurrence among equal distances;
+ *   rounds beyond n give (+inf, -1) (the argmin neutral element, R3/R4).
+ * O(kk * n) by design: this is the repeated reduce the paper describes, not
+ * a selection algorithm.  dist_scratch: n floats; chosen_scratch: n bytes. */
+int orc_nn_knn(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk,
+               float *out_dist, int64_t *out_idx, float *dist_scratch, unsigned char *chosen_scratch) {
+    if (n < 0 || kk < 0 || (n > 0 && (!lat || !lng || !dist_scratch || !chosen_scratch)) ||
+        (kk > 0 && (!out_dist || !out_idx)))
+        return 1;
+    orc_nn_dist(lat, lng, n, q0, q1, dist_scratch);
+    memset(chosen_scratch, 0, (size_t)n);
+    for (int64_t r = 0; r < kk; ++r) {
+        float best = INFINITY;
+        int64_t bi = -1;
+        for (int64_t i = 0; i < n; ++i) {
+            if (chosen_scratch[i]) continue;
+            if (bi < 0 || dist_scratch[i] < best) {  /* strict <: first occurrence wins ties */
+                best = dist_scratch[i];
+                bi = i;
+            }
+        }
+        out_dist[r] = best;
+        out_idx[r] = bi;
+        if (bi >= 0) chosen_scratch[bi] = 1;
+    }
+    return 0;
+}

@@ -208,6 +208,36 @@ def test_library_nn_dist_bitexact_with_numpy_f32():
     assert i == int(np.argmin(want)) and i < 5000  # first copy wins (duplicated data, L1637)
 
 
+def test_golden_nn_knn_hand():
+    g = gold("nn_knn_hand.json")
+    d, i = oracle.nn_knn(np.array(g["lat"], np.float32), np.array(g["lng"], np.float32), g["q"], g["kk"])
+    assert d.tolist() == [float(v) for v in g["dist"]] and i.tolist() == g["idx"]
+
+
+def test_library_nn_knn_is_a_lexicographic_sort():
+    """kk rounds of argmin-with-exclusion = the first kk of the records sorted by
+    (distance, index) (np.lexsort, a different algorithm), incl. the 20x ties (L1637)."""
+    lat, lng, q = workloads.c2_nn(base=3000, reps=20)
+    d0 = lat - np.float32(q[0])
+    d1 = lng - np.float32(q[1])
+    dist = np.sqrt(d0 * d0 + d1 * d1)
+    order = np.lexsort((np.arange(dist.size), dist))
+    for kk in (1, 7, 100, 257):
+        d, i = oracle.nn_knn(lat, lng, q, kk)
+        np.testing.assert_array_equal(i, order[:kk])
+        np.testing.assert_array_equal(d.view(np.uint32), dist[order[:kk]].view(np.uint32))
+    # closed form of the duplication: each distance recurs at stride base, in index order
+    d, i = oracle.nn_knn(lat, lng, q, 60)
+    assert i[:20].tolist() == [int(i[0]) + 3000 * r for r in range(20)]
+    assert np.all(d[:20] == d[0]) and d[20] > d[0]
+    # kk = 1 is the argmin redomap (pinned above); kk > n pads with the neutral element
+    v, j = oracle.redomap(lat, "argmin", "nn_dist", lng, q)
+    assert oracle.nn_knn(lat, lng, q, 1)[1][0] == j
+    d, i = oracle.nn_knn(lat[:5], lng[:5], q, 7)
+    assert sorted(i[:5].tolist()) == list(range(5)) and i[5:].tolist() == [-1, -1]
+    assert np.all(np.isinf(d[5:])) and np.all(np.diff(d[:5]) >= 0)
+
+
 def test_invalid_key_is_rejected():
     with pytest.raises(ValueError):
         oracle.stream_red(np.ones((3, 2), np.float32), np.array([0, 5, 1]), 3)
