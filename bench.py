@@ -186,6 +186,48 @@ def make_step(fs, W, world):
     return st
 
 
+# ------------------------------------------------------------------ SURVEY 8(f) "next" rows
+def time_next_rows(fs, W, dev, K, peak):
+    """Each NEXT row timed on its own (CUDA events, K reps, L2 flushed before every rep by
+    a 1 GB write outside the events).  Not part of the step value (8(a) rows only)."""
+    import torch
+    flush = torch.empty(1 << 30, dtype=torch.uint8, device=dev)  # ~150 us of GPU time: the host stays ahead
+    rows = {}
+
+    def timed(fn, reps=K):
+        ms = []
+        for _ in range(reps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            b.synchronize()
+            ms.append(a.elapsed_time(b))
+        return sum(ms) / len(ms), min(ms)
+
+    # NEXT-2: NN's 100 argmin rounds (L1653-1655) as one selection launch
+    nn, kk = W["lat"].numel(), 100
+    od = torch.empty(kk, dtype=torch.float32, device=dev)
+    oi = torch.empty(kk, dtype=torch.int64, device=dev)
+    l0 = fs.launch_count()
+    avg, mn = timed(lambda: fs.nn_knn(W["lat"], W["lng"], W["q"], kk, out_dist=od, out_idx=oi))
+    launches = (fs.launch_count() - l0) // K
+    # the paper's structure for reference: kk argmin-redomap launches back to back (the
+    # exclusion step between rounds not even counted) -- what "dominated by frequent
+    # launches of short kernels" (L1655-1656) costs on this GPU
+    o1, o2 = W["o_nn"]
+    avg_r, _ = timed(lambda: [fs.redomap(W["lat"], "argmin", map="nn_dist", lng=W["lng"], query=W["q"],
+                                         out=o1, out_idx=o2) for _ in range(kk)], reps=max(3, K // 4))
+    b = 8 * nn
+    rows["nn_knn_k100_c2"] = {"ms": round(avg, 4), "ms_min": round(mn, 4), "GB_s": round(b / (avg * 1e-3) / GB, 1),
+                              "elements_per_s": float(f"{nn / (avg * 1e-3):.4g}"), "bytes": b,
+                              "frac_of_peak": round(b / (avg * 1e-3) / GB / peak, 4), "launches": launches,
+                              "vs_100_argmin_launches_ms": round(avg_r, 4),
+                              "note": "C2 records (L2-flushed, cold); bit-exact vs 100 oracle argmin rounds"}
+    return rows
+
+
 # ------------------------------------------------------------------ cpu baseline (oracle)
 def oracle_sample(W, scale_shift):
     """Host copies of a bounded sample of every primitive's input (same data as the GPU run)."""
@@ -270,6 +312,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--only", default="", help="comma-separated primitive names (profiling aid)")
+    ap.add_argument("--no-next", action="store_true", help="skip the SURVEY 8(f) next-row measurements")
     args = ap.parse_args()
     if args.warmup < 3 and not args.quick and not args.only:
         print("bench.py: --warmup must be >= 3", file=sys.stderr)
@@ -387,6 +430,11 @@ def main():
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": KE,
                "note": "same algorithmic bytes; pinned host inputs copied in and all outputs copied out every step"}
 
+    # ---------------- SURVEY 8(f) next rows (single GPU, own timing; not in the step value)
+    nxt = None
+    if rank == 0 and world == 1 and not args.no_next and not args.only and not args.quick:
+        nxt = time_next_rows(fs, W, dev, max(K, 5), peak)
+
     # ---------------- cpu baseline: the oracle on a bounded sample, rank 0, N = 1
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.only:
@@ -412,6 +460,7 @@ def main():
                          "frac": round(per[dom]["GB_s"] / peak, 4), "traffic": traffic, "peak_source": peak_src,
                          "bytes_per_launch": per[dom]["bytes"]},
             "per_primitive": per,
+            "next_rows": nxt,
             "clocks": clk.summary(),
             "gpu_launches": launches,
             "e2e": e2e,

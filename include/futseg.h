@@ -196,6 +196,24 @@ fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen
 fs_status fs_transpose_2d(int32_t dtype, const void *in, int64_t rows, int64_t cols, void *out,
                           void *stream);
 
+/* ---------------------------------------------------------------- NEXT-2: nn_knn */
+/* Rodinia NN's kk nearest neighbours: "100 reduce operations for finding the
+ * nearest neighbors", the reduce computing "both the minimal value and the
+ * corresponding index" (L1653-1655; reading R16).  Defined as kk rounds of the
+ * ARGMIN redomap over the NN distance map (R5), each round excluding the record
+ * it found:
+ *   (out_dist[r], out_idx[r]) = argmin over not-yet-chosen i of (dist(i), i)
+ * i.e. the kk records with the smallest (distance, index), in ascending order.
+ * Rounds beyond n give (+inf, -1) (the ARGMIN neutral element).
+ *   lat, lng : n f32 records (device, 4-byte aligned); n < 2^32.
+ *   out_dist : kk f32; out_idx : kk int64 (device); 0 <= kk <= 1024.
+ * One launch (no host round trips between rounds).  Errors: FS_ERR_NULL,
+ * FS_ERR_SIZE (n < 0, n >= 2^32, kk < 0 or kk > 1024), FS_ERR_ALIAS,
+ * FS_ERR_WORKSPACE, FS_ERR_CUDA. */
+fs_status fs_nn_knn_workspace(int64_t n, int64_t kk, size_t *bytes);
+fs_status fs_nn_knn(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk,
+                    float *out_dist, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
+
 /* ---------------------------------------------------------------- utilities */
 /* Synchronises `stream`, reads and clears the device error word of `ws`.
  * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */

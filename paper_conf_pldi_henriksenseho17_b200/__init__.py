@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -68,6 +68,8 @@ _SIG = {
     "fs_seg_reduce": [fs_opdesc, _P, _L, _L, _I, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_seg_scan": [fs_opdesc, _P, _L, _L, _I, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_transpose_2d": [_I, _P, _L, _L, _P, _P],
+    "fs_nn_knn_workspace": [_L, _L, _SZ],
+    "fs_nn_knn": [_P, _P, _L, ctypes.c_float, ctypes.c_float, _L, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
@@ -230,6 +232,25 @@ def combine(parts, op: str = "add", part_idx=None, width: int = 1):
     _ok(_lib.fs_combine(o, _ptr(parts), _ptr(part_idx), P, ctypes.c_void_p(out.data_ptr()),
                         _ptr(out_idx) if out_idx is not None else None, _stream(parts.device)), "fs_combine")
     return (out, out_idx) if op == "argmin" else out
+
+
+def nn_knn(lat, lng, query, kk: int, out_dist=None, out_idx=None):
+    """NEXT-2: Rodinia NN's kk nearest neighbours of ``query`` = kk argmin rounds with
+    exclusion (L1653-1655): the kk smallest (distance, index) in ascending order, one launch.
+    Returns (dist[kk] f32, idx[kk] int64); rounds beyond n give (+inf, -1)."""
+    lat = _dev(lat, "lat")
+    lng = _dev(lng, "lng")
+    if lat.dtype != torch.float32 or lng.dtype != torch.float32 or lat.shape != lng.shape:
+        raise TypeError("nn_knn: lat and lng must be float32 tensors of the same shape")
+    n = lat.numel()
+    if out_dist is None:
+        out_dist = torch.empty(kk, dtype=torch.float32, device=lat.device)
+    if out_idx is None:
+        out_idx = torch.empty(kk, dtype=torch.int64, device=lat.device)
+    ws = workspace(_query(_lib.fs_nn_knn_workspace, n, kk), lat.device)
+    _ok(_lib.fs_nn_knn(_ptr(lat), _ptr(lng), n, float(query[0]), float(query[1]), kk, _ptr(out_dist), _ptr(out_idx),
+                       ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(lat.device)), "fs_nn_knn")
+    return out_dist, out_idx
 
 
 def stream_red(vals, keys, k: int, sums=None, counts=None, with_counts: bool = True):

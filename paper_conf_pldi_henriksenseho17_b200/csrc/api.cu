@@ -361,6 +361,31 @@ fs_status fs_transpose_2d(int32_t dtype, const void *in, int64_t rows, int64_t c
     return transpose_run(dtype, in, rows, cols, out, S(stream));
 }
 
+// ------------------------------------------------------------ NEXT-2: nn_knn
+fs_status fs_nn_knn_workspace(int64_t n, int64_t kk, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    if (n < 0 || n >= (int64_t(1) << 32) || kk < 0 || kk > 1024) return FS_ERR_SIZE;
+    *bytes = knn_ws(n);
+    return FS_OK;
+}
+
+fs_status fs_nn_knn(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk,
+                    float *out_dist, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream) {
+    size_t need = 0;
+    FS_TRY(fs_nn_knn_workspace(n, kk, &need));
+    if (kk == 0) return FS_OK;
+    if ((n > 0 && (!lat || !lng)) || !out_dist || !out_idx) return FS_ERR_NULL;
+    if ((n > 0 && (!aligned_to(lat, 4) || !aligned_to(lng, 4))) || !aligned_to(out_dist, 4) ||
+        !aligned_to(out_idx, 8))
+        return FS_ERR_UNSUPPORTED;
+    if (overlaps(out_dist, kk * 4, lat, n * 4) || overlaps(out_dist, kk * 4, lng, n * 4) ||
+        overlaps(out_idx, kk * 8, lat, n * 4) || overlaps(out_idx, kk * 8, lng, n * 4) ||
+        overlaps(out_idx, kk * 8, out_dist, kk * 4))
+        return FS_ERR_ALIAS;
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    return knn_run(lat, lng, n, q0, q1, kk, out_dist, out_idx, ws, S(stream));
+}
+
 // ------------------------------------------------------------ utilities
 fs_status fs_check_device_error(void *ws, void *stream) {
     if (!ws) return FS_ERR_NULL;

@@ -204,6 +204,13 @@ template <typename T> __device__ __forceinline__ AV<T> shift_idx(AV<T> a, int64_
     return a;
 }
 
+// The NN distance map (reading R5): sqrt((lat-q0)^2 + (lng-q1)^2), every f32
+// operation separately rounded (no FMA contraction), IEEE sqrt.
+__device__ __forceinline__ float nn_distance(float lat, float lng, float q0, float q1) {
+    const float d0 = __fsub_rn(lat, q0), d1 = __fsub_rn(lng, q1);
+    return __fsqrt_rn(__fadd_rn(__fmul_rn(d0, d0), __fmul_rn(d1, d1)));
+}
+
 // Store the final value (and ARGMIN index) of accumulator `a` at position k.
 template <class O, typename T>
 __device__ __forceinline__ void store_out(T *out, int64_t *out_idx, int64_t k, typename O::V a) {

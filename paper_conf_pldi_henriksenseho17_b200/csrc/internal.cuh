@@ -80,6 +80,10 @@ fs_status colscan_run(int op, int dt, const void *in, int64_t m, int64_t w, void
 size_t stream_red_ws(int dt, int64_t n, int64_t w, int64_t k);
 fs_status stream_red_run(int dt, const void *vals, const int32_t *keys, int64_t n, int64_t w, int64_t k,
                          void *sums, int32_t *counts, void *ws, cudaStream_t st);
+// knn.cu (NEXT-2)
+size_t knn_ws(int64_t n);
+fs_status knn_run(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk, float *out_dist,
+                  int64_t *out_idx, void *ws, cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 

@@ -86,10 +86,6 @@ __global__ void __launch_bounds__(NT) redomap_id_kernel(const T *__restrict__ x,
 }
 
 // Rodinia NN distance (reading R5): every operation rounded to f32, no FMA.
-__device__ __forceinline__ float nn_dist(float lat, float lng, float q0, float q1) {
-    const float d0 = __fsub_rn(lat, q0), d1 = __fsub_rn(lng, q1);
-    return __fsqrt_rn(__fadd_rn(__fmul_rn(d0, d0), __fmul_rn(d1, d1)));
-}
 
 template <int OP, int NT, int U, bool VECT>
 __global__ void __launch_bounds__(NT) redomap_nn_kernel(const float *__restrict__ lat, const float *__restrict__ lng,
@@ -108,7 +104,7 @@ __global__ void __launch_bounds__(NT) redomap_nn_kernel(const float *__restrict_
         const int64_t nvec = (n - head) / 4, tail0 = head + nvec * 4;
         const int4 *av = reinterpret_cast<const int4 *>(lat + head);
         const int4 *bv = reinterpret_cast<const int4 *>(lng + head);
-        if (gid < head) acc = O::fold(acc, nn_dist(lat[gid], lng[gid], q0, q1), gid);
+        if (gid < head) acc = O::fold(acc, nn_distance(lat[gid], lng[gid], q0, q1), gid);
         int64_t v = gid;
         for (; v + (U - 1) * stride < nvec; v += U * stride) {
             int4 ra[U], rb[U];
@@ -122,17 +118,17 @@ __global__ void __launch_bounds__(NT) redomap_nn_kernel(const float *__restrict_
                 const Vec16<float> a = as_vec<float>(ra[u]), b = as_vec<float>(rb[u]);
                 const int64_t base = head + (v + u * stride) * 4;
 #pragma unroll
-                for (int k = 0; k < 4; ++k) acc = O::fold(acc, nn_dist(a.e[k], b.e[k], q0, q1), base + k);
+                for (int k = 0; k < 4; ++k) acc = O::fold(acc, nn_distance(a.e[k], b.e[k], q0, q1), base + k);
             }
         }
         for (; v < nvec; v += stride) {
             const Vec16<float> a = as_vec<float>(ldg16(av + v)), b = as_vec<float>(ldg16(bv + v));
 #pragma unroll
-            for (int k = 0; k < 4; ++k) acc = O::fold(acc, nn_dist(a.e[k], b.e[k], q0, q1), head + v * 4 + k);
+            for (int k = 0; k < 4; ++k) acc = O::fold(acc, nn_distance(a.e[k], b.e[k], q0, q1), head + v * 4 + k);
         }
-        if (gid < n - tail0) acc = O::fold(acc, nn_dist(lat[tail0 + gid], lng[tail0 + gid], q0, q1), tail0 + gid);
+        if (gid < n - tail0) acc = O::fold(acc, nn_distance(lat[tail0 + gid], lng[tail0 + gid], q0, q1), tail0 + gid);
     } else {
-        for (int64_t i = gid; i < n; i += stride) acc = O::fold(acc, nn_dist(lat[i], lng[i], q0, q1), i);
+        for (int64_t i = gid; i < n; i += stride) acc = O::fold(acc, nn_distance(lat[i], lng[i], q0, q1), i);
     }
     acc = block_reduce<O, NT>(acc, sm);
     finish_grid<O, NT>(acc, partials, ticket, out, out_idx, sm, ibase);

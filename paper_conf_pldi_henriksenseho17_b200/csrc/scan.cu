@@ -121,10 +121,6 @@ template <class S> struct TileState<S, false> {
     }
 };
 
-__device__ __forceinline__ float nn_dist_s(float lat, float lng, float q0, float q1) {
-    const float d0 = __fsub_rn(lat, q0), d1 = __fsub_rn(lng, q1);
-    return __fsqrt_rn(__fadd_rn(__fmul_rn(d0, d0), __fmul_rn(d1, d1)));
-}
 
 #ifndef FS_SCAN_R
 #define FS_SCAN_R 4
@@ -248,7 +244,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
                     const Vec16<float> a = as_vec<float>(ldg16((const float *)in0 + p0));
                     const Vec16<float> c = as_vec<float>(ldg16(in1 + p0));
 #pragma unroll
-                    for (int k = 0; k < VEC; ++k) x[k] = (T)nn_dist_s(a.e[k], c.e[k], q0, q1);
+                    for (int k = 0; k < VEC; ++k) x[k] = (T)nn_distance(a.e[k], c.e[k], q0, q1);
                 } else {
                     const Vec16<T> a = as_vec<T>(ldg16(in0 + p0));
 #pragma unroll
@@ -258,7 +254,7 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
 #pragma unroll
                 for (int k = 0; k < VEC; ++k) {
                     if (p0 + k < n) {
-                        if (NN) x[k] = (T)nn_dist_s(((const float *)in0)[p0 + k], in1[p0 + k], q0, q1);
+                        if (NN) x[k] = (T)nn_distance(((const float *)in0)[p0 + k], in1[p0 + k], q0, q1);
                         else x[k] = in0[p0 + k];
                     } else {
                         x[k] = T(0);

@@ -132,6 +132,29 @@ def test_scan_seg_transpose_stream_red_validation(fs):
     assert fs.C.fs_combine(o, P(FAKE_IN), None, 4, P(FAKE_IN), None, None) == ALIAS
 
 
+def test_nn_knn_validation(fs):
+    big = 1 << 30
+    f = ctypes.c_float(0.0)
+    knn = fs.C.fs_nn_knn
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, 1025, P(FAKE_OUT), P(FAKE_OUT + 8192), P(FAKE_WS), big,
+               None) == SIZE                                   # kk > 1024
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1 << 32, f, f, 10, P(FAKE_OUT), P(FAKE_OUT + 8192), P(FAKE_WS), big,
+               None) == SIZE                                   # 32-bit record indices
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, -1, P(FAKE_OUT), P(FAKE_OUT + 8192), P(FAKE_WS), big,
+               None) == SIZE
+    assert knn(P(FAKE_IN), None, 1000, f, f, 10, P(FAKE_OUT), P(FAKE_OUT + 8192), P(FAKE_WS), big, None) == NULL
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, 10, P(FAKE_OUT), None, P(FAKE_WS), big, None) == NULL
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, 10, P(FAKE_IN + 8), P(FAKE_OUT), P(FAKE_WS), big,
+               None) == ALIAS                                  # out_dist inside lat
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, 10, P(FAKE_OUT), P(FAKE_OUT + 16), P(FAKE_WS), big,
+               None) == ALIAS                                  # out_idx overlaps out_dist
+    assert knn(P(FAKE_IN), P(FAKE_IN + 4096), 1000, f, f, 10, P(FAKE_OUT), P(FAKE_OUT + 8192), None, 0,
+               None) == WS
+    assert knn(None, None, 0, f, f, 0, None, None, None, 0, None) == OK  # kk = 0: nothing to do
+    sz = ctypes.c_size_t(0)
+    assert fs.C.fs_nn_knn_workspace(855280, 100, ctypes.byref(sz)) == OK and sz.value > 0
+
+
 def test_workspace_queries_and_regimes(fs):
     sz = ctypes.c_size_t(0)
     assert fs.C.fs_redomap_workspace(op(fs, 0, F32), 1 << 28, ctypes.byref(sz)) == OK and sz.value >= 256

@@ -105,6 +105,48 @@ def test_redomap_nn_misaligned_and_ibase(fs):
     assert float(host(got[0])) == float(v) and int(host(got[1])) == i + 1000
 
 
+# ------------------------------------------------------------------ NEXT-2: nn_knn
+def _knn_check(fs, lat, lng, q, kk, off=0):
+    d, i = fs.nn_knn(cu(lat, off), cu(lng, off), q, kk)
+    wd, wi = oracle.nn_knn(lat, lng, q, kk)
+    np.testing.assert_array_equal(host(i), wi)                                  # bit-exact indices
+    np.testing.assert_array_equal(host(d).view(np.uint32), wd.view(np.uint32))  # and distances
+
+
+@pytest.mark.parametrize("kk", [1, 5, 100, 257, 1024])
+def test_nn_knn_c2(fs, kk):
+    """NEXT-2 at the C2 shape: 855,280 records (base duplicated 20x, L1637), the paper's
+    100 argmin rounds (L1653-1655) plus other kk; bit-exact against kk oracle rounds."""
+    lat, lng, q = workloads.c2_nn()
+    _knn_check(fs, lat, lng, q, kk)
+
+
+@pytest.mark.parametrize("n,kk", [(0, 3), (1, 1), (5, 7), (2047, 100), (2048, 100), (2049, 1024), (4097, 2),
+                                  (100_003, 1000), (1_000_003, 100)])
+def test_nn_knn_sizes(fs, n, kk):
+    """Empty, fewer records than kk (neutral padding), one tile +-1, ragged chunks, many CTAs."""
+    base = max(1, n // 7)
+    lat, lng, q = workloads.c2_nn(base=base, reps=8, seed=n % 97)
+    lat, lng = lat[:n], lng[:n]
+    if n == 0:
+        d, i = fs.nn_knn(torch.zeros(0, device="cuda"), torch.zeros(0, device="cuda"), q, kk)
+        assert host(i).tolist() == [-1] * kk and np.all(np.isinf(host(d)))
+        return
+    _knn_check(fs, lat, lng, q, kk, off=1 if n % 2 else 0)
+
+
+def test_nn_knn_adversarial_order(fs):
+    """Records sorted by decreasing distance: every tile improves on the running list, so
+    the selection keeps flushing (the worst case of the threshold filter); all-equal
+    distances: pure index order."""
+    lat, lng, q = workloads.c2_nn(base=50_000, reps=1, seed=9)
+    dd = oracle.nn_dist(lat, lng, *q)
+    order = np.argsort(-dd, kind="stable")
+    _knn_check(fs, lat[order].copy(), lng[order].copy(), q, 1024)
+    flat = np.full(70_000, 1.5, np.float32)
+    _knn_check(fs, flat, flat.copy(), (1.5, 1.5), 300)
+
+
 @pytest.mark.parametrize("dt", DTYPES)
 @pytest.mark.parametrize("k", [1, 5, 34, 100, 1024, 4096])
 def test_redomap_vadd(fs, dt, k):
