@@ -60,8 +60,9 @@ def _L():
         lib.orc_stream_red.argtypes = [I, P, P, L, L, L, P, P]
         lib.orc_transpose.argtypes = [L, P, L, L, P]
         lib.orc_nn_knn.argtypes = [P, P, L, ctypes.c_float, ctypes.c_float, L, P, P, P, P]
+        lib.orc_kmeans_step.argtypes = [P, L, L, P, L, P, P, P, P, P, P]
         for f in ("orc_reduce", "orc_scan", "orc_nn_dist", "orc_vreduce", "orc_seg_reduce",
-                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn"):
+                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn", "orc_kmeans_step"):
             getattr(lib, f).restype = I
         _lib = lib
     return _lib
@@ -128,6 +129,27 @@ def nn_knn(lat, lng, q, kk):
     _check(_L().orc_nn_knn(_p(lat), _p(lng), n, float(q[0]), float(q[1]), kk, _p(dist), _p(idx), _p(ds), _p(ch)),
            "nn_knn")
     return dist, idx
+
+
+def kmeans_step(points, centres, prev=None):
+    """NEXT-1: one Rodinia K-means iteration (Sec. 2.4; readings R18/R19):
+    f32 fma distance argmin (first centre on ties), f64 sums, counts, new centres
+    (old centre kept for an empty cluster), delta vs ``prev``.
+    Returns (membership[n] i32, sums[k][d] f64, counts[k] i32, new_centres[k][d] f64, delta)."""
+    points = np.ascontiguousarray(points, np.float32)
+    centres = np.ascontiguousarray(centres, np.float32)
+    n, d = points.shape
+    k = centres.shape[0]
+    assert centres.shape[1] == d
+    mem = np.zeros(max(n, 1), np.int32)
+    sums = np.zeros((k, d), np.float64)
+    counts = np.zeros(k, np.int32)
+    newc = np.zeros((k, d), np.float64)
+    delta = np.zeros(1, np.int64)
+    pv = None if prev is None else np.ascontiguousarray(prev, np.int32)
+    _check(_L().orc_kmeans_step(_p(points), n, d, _p(centres), k, _p(pv) if pv is not None else None, _p(mem),
+                                _p(sums), _p(counts), _p(newc), _p(delta)), "kmeans_step")
+    return mem[:n], sums, counts, newc, int(delta[0])
 
 
 def redomap(x, op="add", map="id", lng=None, q=(0.0, 0.0)):

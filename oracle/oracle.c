@@ -288,3 +288,49 @@ int orc_nn_knn(const float *lat, const float *lng, int64_t n, float q0, float q1
     }
     return 0;
 }
+
+/* NEXT-1, one iteration of Rodinia's K-means (Sec. 2.4; Fig 4; L1628-1649):
+ *   assignment  membership[i] = argmin_c E(i, c), the first c on ties (R3), with
+ *               E(i, c) = sum over j = 0..d-1, in order, of (x_ij - c_cj)^2 computed
+ *               in f32 as acc = fmaf(t, t, acc), t = x_ij - c_cj (reading R18:
+ *               Rodinia's squared Euclidean distance, one rounding per fma);
+ *   new centres sums[c][j] = sum of x_ij over membership[i] == c (f64, R2),
+ *               counts[c]; new_centres[c][j] = sums/counts when counts > 0, else
+ *               the old centre (reading R19) -- the segmented reduction of L1649;
+ *   delta       #{ i : membership[i] != prev[i] } (Rodinia's convergence test),
+ *               only if prev != NULL.
+ * Straight loops in index order; sums/new_centres are f64.  */
+int orc_kmeans_step(const float *x, int64_t n, int64_t d, const float *cen, int64_t k, const int32_t *prev,
+                    int32_t *membership, double *sums, int32_t *counts, double *new_cen, int64_t *delta) {
+    if (n < 0 || d < 1 || k < 1 || (n > 0 && (!x || !membership)) || !cen || !sums || !counts || !new_cen)
+        return 1;
+    int64_t changed = 0;
+    for (int64_t c = 0; c < k; ++c) {
+        counts[c] = 0;
+        for (int64_t j = 0; j < d; ++j) sums[c * d + j] = 0.0;
+    }
+    for (int64_t i = 0; i < n; ++i) {
+        float best = 0.0f;
+        int32_t bc = -1;
+        for (int64_t c = 0; c < k; ++c) {
+            float acc = 0.0f;
+            for (int64_t j = 0; j < d; ++j) {
+                const float t = x[i * d + j] - cen[c * d + j];
+                acc = fmaf(t, t, acc);
+            }
+            if (bc < 0 || acc < best) { /* strict <: first centre wins ties */
+                best = acc;
+                bc = (int32_t)c;
+            }
+        }
+        membership[i] = bc;
+        if (prev && prev[i] != bc) ++changed;
+        counts[bc] += 1;
+        for (int64_t j = 0; j < d; ++j) sums[bc * d + j] += (double)x[i * d + j];
+    }
+    for (int64_t c = 0; c < k; ++c)
+        for (int64_t j = 0; j < d; ++j)
+            new_cen[c * d + j] = counts[c] > 0 ? sums[c * d + j] / (double)counts[c] : (double)cen[c * d + j];
+    if (delta) *delta = prev ? changed : 0;
+    return 0;
+}

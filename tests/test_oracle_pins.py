@@ -238,6 +238,61 @@ def test_library_nn_knn_is_a_lexicographic_sort():
     assert np.all(np.isinf(d[5:])) and np.all(np.diff(d[:5]) >= 0)
 
 
+def test_golden_kmeans_step_hand():
+    g = gold("kmeans_step_hand.json")
+    m, sums, counts, newc, delta = oracle.kmeans_step(np.array(g["points"], np.float32),
+                                                      np.array(g["centres"], np.float32), np.array(g["prev"]))
+    assert m.tolist() == g["membership"] and counts.tolist() == g["counts"] and delta == g["delta"]
+    assert sums.tolist() == g["sums"]
+    np.testing.assert_allclose(newc, g["new_centres"], rtol=1e-15)
+
+
+def test_kmeans_step_against_float64_brute_force():
+    """Assignment: the f32 fma distance argmin is the float64 argmin except at f32-level
+    near-ties, where it is still a valid minimum; centre update = numpy bincount / add.at /
+    mean (library routines); the empty cluster keeps its centre; delta = changed labels."""
+    r = np.random.default_rng(17)
+    x = r.random((20_000, 34)).astype(np.float32)
+    cen = x[r.choice(x.shape[0], 31, replace=False)].copy()
+    cen = np.concatenate([cen, np.full((1, 34), 50.0, np.float32)])  # far away: stays empty
+    prev = r.integers(0, 32, x.shape[0]).astype(np.int32)
+    m, sums, counts, newc, delta = oracle.kmeans_step(x, cen, prev)
+    e64 = ((x.astype(np.float64)[:, None, :] - cen.astype(np.float64)[None]) ** 2).sum(-1)
+    best = e64.min(1)
+    assert np.all(e64[np.arange(x.shape[0]), m] <= best * (1 + 1e-5))
+    assert np.mean(m == e64.argmin(1)) > 0.999
+    np.testing.assert_array_equal(counts, np.bincount(m, minlength=32))
+    want = np.zeros((32, 34))
+    np.add.at(want, m, x.astype(np.float64))
+    np.testing.assert_allclose(sums, want, rtol=1e-12)
+    assert counts[31] == 0 and np.all(newc[31] == 50.0)
+    for c in range(31):
+        np.testing.assert_allclose(newc[c], x[m == c].astype(np.float64).mean(0), rtol=1e-12)
+    assert delta == int(np.count_nonzero(m != prev))
+
+
+def test_kmeans_step_closed_forms():
+    r = np.random.default_rng(5)
+    x = r.random((500, 7)).astype(np.float32)
+    # centres taken from the points: those points are at distance exactly 0
+    idx = np.array([3, 100, 250, 499])
+    m, *_ = oracle.kmeans_step(x, x[idx])
+    assert m[idx].tolist() == [0, 1, 2, 3]
+    # a duplicated centre never wins (ties go to the first)
+    cen = np.concatenate([x[idx], x[idx[:1]]])
+    m2, _, counts, _, _ = oracle.kmeans_step(x, cen)
+    assert counts[4] == 0 and np.array_equal(m2, m)
+    # k = 1: every point in cluster 0; the new centre is the column mean; no prev -> delta 0
+    m1, s1, c1, n1, d1 = oracle.kmeans_step(x, x[:1])
+    assert np.all(m1 == 0) and c1.tolist() == [500] and d1 == 0
+    np.testing.assert_allclose(n1[0], x.astype(np.float64).mean(0), rtol=1e-12)
+    # banana split / Fig 4c: the centre sums are stream_red over the new membership
+    s_sr, c_sr = oracle.stream_red(x, m, 4)
+    _, s_k, c_k, _, _ = oracle.kmeans_step(x, x[idx])
+    np.testing.assert_array_equal(c_sr, c_k)
+    np.testing.assert_allclose(s_sr, s_k, rtol=1e-12)
+
+
 def test_invalid_key_is_rejected():
     with pytest.raises(ValueError):
         oracle.stream_red(np.ones((3, 2), np.float32), np.array([0, 5, 1]), 3)
