@@ -225,6 +225,29 @@ def time_next_rows(fs, W, dev, K, peak):
                               "frac_of_peak": round(b / (avg * 1e-3) / GB / peak, 4), "launches": launches,
                               "vs_100_argmin_launches_ms": round(avg_r, 4),
                               "note": "C2 records (L2-flushed, cold); bit-exact vs 100 oracle argmin rounds"}
+    # NEXT-1: one fused K-means iteration at C5 (n = 2^26, d = 34, k = 32): assignment on the
+    # tensor cores (TF32, certified exact) + stream_red centre update + new centres + delta
+    pts = W["pts"]
+    kn, d = pts.shape
+    g = torch.Generator(device=dev).manual_seed(77)
+    cen = pts[torch.randint(0, kn, (32,), device=dev, generator=g)].clone()
+    prev = W["mem"]
+    mem = torch.empty(kn, dtype=torch.int32, device=dev)
+    sums = torch.empty((32, d), dtype=torch.float32, device=dev)
+    cnt = torch.empty(32, dtype=torch.int32, device=dev)
+    newc = torch.empty((32, d), dtype=torch.float32, device=dev)
+    dl = torch.empty(1, dtype=torch.int64, device=dev)
+    avg, mn = timed(lambda: fs.kmeans_step(pts, cen, prev=prev, membership=mem, sums=sums, counts=cnt,
+                                           new_centres=newc, delta=dl))
+    b = kn * (4 * d + 4 + 4)  # points + prev membership in, new membership out
+    flops = 2.0 * kn * 32 * d  # the x.c contraction (what the tensor cores do)
+    rows["kmeans_step_c5_k32_d34"] = {"ms": round(avg, 4), "ms_min": round(mn, 4),
+                                      "GB_s": round(b / (avg * 1e-3) / GB, 1),
+                                      "elements_per_s": float(f"{kn / (avg * 1e-3):.4g}"), "bytes": b,
+                                      "frac_of_peak": round(b / (avg * 1e-3) / GB / peak, 4),
+                                      "tflops_tf32": round(flops / (avg * 1e-3) / 1e12, 1),
+                                      "note": "fused assignment (mma.sync TF32 + exact near-tie re-evaluation) + "
+                                              "stream_red + new centres + delta; membership bit-exact vs f32 oracle"}
     return rows
 
 

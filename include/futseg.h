@@ -214,6 +214,26 @@ fs_status fs_nn_knn_workspace(int64_t n, int64_t kk, size_t *bytes);
 fs_status fs_nn_knn(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk,
                     float *out_dist, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
 
+/* ---------------------------------------------------------------- NEXT-1: kmeans_step */
+/* One fused iteration of Rodinia's K-means (Sec. 2.4; the
+ * assignment map fused into the centre stream_red, F6 L1075-1090):
+ *   membership[i]  = argmin_c E(i, c), the first c on ties            (R3, R18)
+ *   E(i, c)        = sum_j (x_ij - c_cj)^2 in f32, j in order, acc = fma(t, t, acc),
+ *                    t = x_ij - c_cj (exactly this f32 sequence: membership is
+ *                    bit-exact; the tensor-core ranking is certified by an error
+ *                    bound and re-evaluated exactly for near-ties)
+ *   sums[c][j]     = sum of x_ij over membership[i] == c, counts[c]   (Fig 4c)
+ *   new_centres    = sums / counts; an empty cluster keeps its centre (R19)
+ *   *delta         = #{ i : membership[i] != prev[i] } (0 when prev is NULL)
+ *   points  : [n][d] f32 row-major, 16-byte aligned; centres : [k][d] f32.
+ *   prev, membership, new_centres, delta : optional (NULL).
+ *   1 <= k <= 32, 1 <= d <= 40 (else FS_ERR_UNSUPPORTED); n >= 0.
+ * Outputs are overwritten; they must not overlap the inputs (FS_ERR_ALIAS). */
+fs_status fs_kmeans_step_workspace(int64_t n, int64_t d, int64_t k, size_t *bytes);
+fs_status fs_kmeans_step(const float *points, int64_t n, int64_t d, const float *centres, int64_t k,
+                         const int32_t *prev, int32_t *membership, float *sums, int32_t *counts,
+                         float *new_centres, int64_t *delta, void *ws, size_t ws_bytes, void *stream);
+
 /* ---------------------------------------------------------------- utilities */
 /* Synchronises `stream`, reads and clears the device error word of `ws`.
  * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */

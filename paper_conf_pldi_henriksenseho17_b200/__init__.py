@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "kmeans_step", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -70,6 +70,8 @@ _SIG = {
     "fs_transpose_2d": [_I, _P, _L, _L, _P, _P],
     "fs_nn_knn_workspace": [_L, _L, _SZ],
     "fs_nn_knn": [_P, _P, _L, ctypes.c_float, ctypes.c_float, _L, _P, _P, _P, ctypes.c_size_t, _P],
+    "fs_kmeans_step_workspace": [_L, _L, _L, _SZ],
+    "fs_kmeans_step": [_P, _L, _L, _P, _L, _P, _P, _P, _P, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
@@ -251,6 +253,37 @@ def nn_knn(lat, lng, query, kk: int, out_dist=None, out_idx=None):
     _ok(_lib.fs_nn_knn(_ptr(lat), _ptr(lng), n, float(query[0]), float(query[1]), kk, _ptr(out_dist), _ptr(out_idx),
                        ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(lat.device)), "fs_nn_knn")
     return out_dist, out_idx
+
+
+def kmeans_step(points, centres, prev=None, membership=None, sums=None, counts=None, new_centres=None,
+                delta=None, with_membership: bool = True):
+    """NEXT-1: one fused Rodinia K-means iteration (Sec. 2.4; F6 fusion):
+    assignment (first centre on ties) + stream_red centre sums/counts + new centres.
+    points [n][d] f32 (16-byte aligned), centres [k][d] f32; k <= 32, d <= 40.
+    Returns (membership [n] i32 or None, sums [k][d], counts [k], new_centres [k][d],
+    delta (1-element int64 tensor; 0 without prev))."""
+    points = _dev(points, "points")
+    centres = _dev(centres, "centres")
+    if points.dtype != torch.float32 or centres.dtype != torch.float32 or points.dim() != 2 or centres.dim() != 2:
+        raise TypeError("kmeans_step: points [n][d] and centres [k][d] must be float32 matrices")
+    n, d = points.shape
+    k = centres.shape[0]
+    if centres.shape[1] != d:
+        raise ValueError("kmeans_step: centres must have the points' width")
+    dev = points.device
+    if prev is not None:
+        prev = _dev(prev, "prev")
+    if membership is None and with_membership:
+        membership = torch.empty(n, dtype=torch.int32, device=dev)
+    sums = torch.empty((k, d), dtype=torch.float32, device=dev) if sums is None else sums
+    counts = torch.empty(k, dtype=torch.int32, device=dev) if counts is None else counts
+    new_centres = torch.empty((k, d), dtype=torch.float32, device=dev) if new_centres is None else new_centres
+    delta = torch.empty(1, dtype=torch.int64, device=dev) if delta is None else delta
+    ws = workspace(_query(_lib.fs_kmeans_step_workspace, n, d, k), dev)
+    _ok(_lib.fs_kmeans_step(_ptr(points), n, d, _ptr(centres), k, _ptr(prev), _ptr(membership), _ptr(sums),
+                            _ptr(counts), _ptr(new_centres), _ptr(delta), ctypes.c_void_p(ws.data_ptr()), ws.numel(),
+                            _stream(dev)), "fs_kmeans_step")
+    return membership, sums, counts, new_centres, delta
 
 
 def stream_red(vals, keys, k: int, sums=None, counts=None, with_counts: bool = True):

@@ -386,6 +386,41 @@ fs_status fs_nn_knn(const float *lat, const float *lng, int64_t n, float q0, flo
     return knn_run(lat, lng, n, q0, q1, kk, out_dist, out_idx, ws, S(stream));
 }
 
+// ------------------------------------------------------------ NEXT-1: kmeans_step
+fs_status fs_kmeans_step_workspace(int64_t n, int64_t d, int64_t k, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    if (n < 0 || mul_overflows(n, d) || mul_overflows(n * (d > 0 ? d : 1), 4)) return FS_ERR_SIZE;
+    if (k < 1 || k > 32 || d < 1 || d > 40) return FS_ERR_UNSUPPORTED;
+    *bytes = kmeans_ws(n, d, k);
+    return FS_OK;
+}
+
+fs_status fs_kmeans_step(const float *points, int64_t n, int64_t d, const float *centres, int64_t k,
+                         const int32_t *prev, int32_t *membership, float *sums, int32_t *counts, float *new_centres,
+                         int64_t *delta, void *ws, size_t ws_bytes, void *stream) {
+    size_t need = 0;
+    FS_TRY(fs_kmeans_step_workspace(n, d, k, &need));
+    if ((n > 0 && !points) || !centres || !sums || !counts) return FS_ERR_NULL;
+    if ((n > 0 && !aligned_to(points, 16)) || !aligned_to(centres, 4) || !aligned_to(sums, 4) ||
+        !aligned_to(counts, 4) || (prev && !aligned_to(prev, 4)) || (membership && !aligned_to(membership, 4)) ||
+        (new_centres && !aligned_to(new_centres, 4)) || (delta && !aligned_to(delta, 8)))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t pb = n * d * 4, cb = k * d * 4;
+    const void *ins[3] = {points, centres, prev};
+    const int64_t inb[3] = {pb, cb, n * 4};
+    void *outs[5] = {membership, sums, counts, new_centres, delta};
+    const int64_t outb[5] = {n * 4, cb, k * 4, cb, 8};
+    for (int o = 0; o < 5; ++o) {
+        if (!outs[o]) continue;
+        for (int i = 0; i < 3; ++i)
+            if (ins[i] && overlaps(outs[o], outb[o], ins[i], inb[i])) return FS_ERR_ALIAS;
+        for (int p = 0; p < o; ++p)
+            if (outs[p] && overlaps(outs[o], outb[o], outs[p], outb[p])) return FS_ERR_ALIAS;
+    }
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    return kmeans_run(points, n, d, centres, k, prev, membership, sums, counts, new_centres, delta, ws, S(stream));
+}
+
 // ------------------------------------------------------------ utilities
 fs_status fs_check_device_error(void *ws, void *stream) {
     if (!ws) return FS_ERR_NULL;

@@ -84,6 +84,11 @@ fs_status stream_red_run(int dt, const void *vals, const int32_t *keys, int64_t 
 size_t knn_ws(int64_t n);
 fs_status knn_run(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk, float *out_dist,
                   int64_t *out_idx, void *ws, cudaStream_t st);
+// kmeans.cu (NEXT-1)
+size_t kmeans_ws(int64_t n, int64_t d, int64_t k);
+fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, int64_t k, const int32_t *prev,
+                     int32_t *membership, float *sums, int32_t *counts, float *new_cen, int64_t *delta, void *ws,
+                     cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 

@@ -155,6 +155,31 @@ def test_nn_knn_validation(fs):
     assert fs.C.fs_nn_knn_workspace(855280, 100, ctypes.byref(sz)) == OK and sz.value > 0
 
 
+def test_kmeans_step_validation(fs):
+    big = 1 << 30
+    km = fs.C.fs_kmeans_step
+    A = lambda o: P(FAKE_OUT + o)
+    ok_args = lambda: [P(FAKE_IN), 1000, 34, P(FAKE_IN + (1 << 20)), 32, None, A(0), A(1 << 16), A(1 << 17),
+                       A(1 << 18), A(1 << 19), P(FAKE_WS), big, None]
+    a = ok_args(); a[4] = 33
+    assert km(*a) == UNSUP                                    # k > 32
+    a = ok_args(); a[2] = 41
+    assert km(*a) == UNSUP                                    # d > 40
+    a = ok_args(); a[0] = P(FAKE_IN + 4)
+    assert km(*a) == UNSUP                                    # points must be 16-byte aligned (TMA)
+    a = ok_args(); a[7] = None
+    assert km(*a) == NULL                                     # sums required
+    a = ok_args(); a[6] = P(FAKE_IN + 64)
+    assert km(*a) == ALIAS                                    # membership inside the points
+    a = ok_args(); a[8] = A(1 << 16)
+    assert km(*a) == ALIAS                                    # counts on top of sums
+    a = ok_args(); a[11] = None; a[12] = 0
+    assert km(*a) == WS
+    sz = ctypes.c_size_t(0)
+    assert fs.C.fs_kmeans_step_workspace(1 << 26, 34, 32, ctypes.byref(sz)) == OK and sz.value > 0
+    assert fs.C.fs_kmeans_step_workspace(-1, 34, 32, ctypes.byref(sz)) == SIZE
+
+
 def test_workspace_queries_and_regimes(fs):
     sz = ctypes.c_size_t(0)
     assert fs.C.fs_redomap_workspace(op(fs, 0, F32), 1 << 28, ctypes.byref(sz)) == OK and sz.value >= 256

@@ -105,6 +105,51 @@ def test_redomap_nn_misaligned_and_ibase(fs):
     assert float(host(got[0])) == float(v) and int(host(got[1])) == i + 1000
 
 
+# ------------------------------------------------------------------ NEXT-1: kmeans_step
+def _km_check(fs, pts, cen, prev=None, tag=""):
+    m, sums, counts, newc, delta = fs.kmeans_step(cu(pts), cu(cen), prev=cu(prev) if prev is not None else None)
+    wm, ws, wc, wn, wd = oracle.kmeans_step(pts, cen, prev)
+    np.testing.assert_array_equal(host(m), wm)                 # bit-exact assignment
+    np.testing.assert_array_equal(host(counts), wc)
+    assert int(host(delta)[0]) == wd
+    absum = np.zeros_like(ws)
+    np.add.at(absum, wm, np.abs(pts).astype(np.float64))
+    assert_reduced(sums, ws, "add", absum, f"kmeans sums {tag}")
+    got_n = host(newc).astype(np.float64)
+    scale = np.where(wc[:, None] > 0, absum / np.maximum(wc[:, None], 1), np.abs(cen))
+    assert np.all(np.abs(got_n - wn) <= 1e-4 * scale + 1e-30), f"kmeans new centres {tag}"
+
+
+@pytest.mark.parametrize("d,k", [(34, 5), (34, 32), (1, 3), (8, 8), (33, 17), (40, 32), (17, 1), (2, 32)])
+def test_kmeans_step_shapes(fs, d, k):
+    """Random centres picked from the points (so many near-ties on small d): membership
+    bit-exact vs the f32 oracle, counts exact, sums/new centres within 1e-4."""
+    r = np.random.default_rng(d * 100 + k)
+    n = 50_021
+    pts = r.random((n, d)).astype(np.float32)
+    cen = pts[r.choice(n, k, replace=False)].copy()
+    prev = r.integers(0, k, n).astype(np.int32)
+    _km_check(fs, pts, cen, prev, f"d={d} k={k}")
+
+
+def test_kmeans_step_c3_kdd_and_ties(fs):
+    """kdd_cup shape (BASELINE configs[2]: n=494,019, d=34, k=5) with clustered points;
+    duplicated centres (exact ties: the first wins) and an empty far-away cluster;
+    signed data; a few points only; a second iteration from the new centres."""
+    pts, mem = workloads.c3_kmeans(keys="clustered")
+    cen = pts[:5].copy()
+    m, _, _, newc, _ = fs.kmeans_step(cu(pts), cu(cen))
+    _km_check(fs, pts, cen, None, "c3")
+    _km_check(fs, pts, host(newc), host(m), "c3 iteration 2")
+    dup = np.concatenate([cen, cen[:2], np.full((1, 34), 1e3, np.float32)])
+    _km_check(fs, pts, dup, None, "duplicated + empty")
+    sg = workloads.mixed((30_000, 34), 3, np.float32) * 100
+    _km_check(fs, sg, sg[:32].copy(), None, "signed")
+    for n in (0, 1, 15, 16, 17, 100):
+        small = pts[:n].copy()
+        _km_check(fs, small, cen, None, f"n={n}")
+
+
 # ------------------------------------------------------------------ NEXT-2: nn_knn
 def _knn_check(fs, lat, lng, q, kk, off=0):
     d, i = fs.nn_knn(cu(lat, off), cu(lng, off), q, kk)
