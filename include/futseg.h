@@ -247,6 +247,10 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *   4 = column kernel (FS_COL_MAJOR: thread per segment, coalesced rows)
  *   5 = single-pass segmented look-back scan (fs_seg_scan, FS_ROW_MAJOR)
  *   6 = empty input (neutral fill)
+ *   7 = KS0 fs_seg_scan of power-of-two rows up to 256 16-byte vectors (seglen <=
+ *       256 * 16/sizeof(elem), FS_ROW_MAJOR, 16-byte aligned buffers; others take 5):
+ *       in-register scan, shuffle scan across the lanes of a segment and, for rows
+ *       longer than a warp's 32 vectors, a shared-memory combine across its warps
  * Returns -1 for invalid arguments. */
 int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen,
                       int32_t layout);

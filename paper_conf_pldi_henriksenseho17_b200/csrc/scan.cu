@@ -1437,6 +1437,148 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
 
 static size_t scan_state_bytes(int64_t ntiles) { return align_up((size_t)ntiles * 8, 256); }
 
+// ---------------------------------------------------------------- KS0: short power-of-two segments
+// seg_scan for regular segments of length L = 2^j <= 32 * VEC with 16-byte aligned
+// buffers.  A 16-byte vector never straddles a segment boundary unless L < VEC, and a
+// segment of L > VEC elements is G = L / VEC consecutive vectors, i.e. G consecutive
+// lanes of one warp (the grid-stride order maps vector v to lane v mod 32).  So the
+// segmented scan needs no look-back and no segment flags at all: an in-register scan of
+// the lane's vector, then an inclusive shuffle scan of the lane totals within each
+// G-lane group (log2 G steps) and one (+) per element.  One read and one write per
+// element, like a copy.
+template <int OP, typename T, int U>
+__global__ void __launch_bounds__(256)
+segscan_vec_kernel(const T *__restrict__ x, int64_t n, int L, int G, T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    const int lane = threadIdx.x & 31, lg = lane & (G - 1);
+    const int64_t nvec = n / VEC;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t gid0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t iters = (nvec + stride - 1) / stride;  // warp-uniform: every lane shuffles
+    for (int64_t it0 = 0; it0 < iters; it0 += U) {
+        int4 r[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            if (it0 + u < iters && v < nvec) r[u] = ldg16(x + v * VEC);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = gid0 + (it0 + u) * stride;
+            const bool ok = it0 + u < iters && v < nvec;
+            if (it0 + u >= iters) break;  // warp-uniform
+            const Vec16<T> e = as_vec<T>(r[u]);
+            V a[VEC];
+            if (L <= VEC) {  // whole segments inside the vector
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) {
+                    const int j = k & (L - 1);  // segment-local index
+                    a[k] = j == 0 ? O::lift(e.e[k], 0) : O::fold(a[k > 0 ? k - 1 : 0], e.e[k], j);
+                }
+            } else {
+                const int j0 = lg * VEC;  // segment-local index of the vector's first element
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) a[k] = k == 0 ? O::lift(e.e[0], j0) : O::fold(a[k - 1], e.e[k], j0 + k);
+                V incl = ok ? a[VEC - 1] : O::id();
+#pragma unroll 1
+                for (int dd = 1; dd < G; dd <<= 1) {
+                    const V y = shfl_up(incl, dd);
+                    if (lg >= dd) incl = O::comb(y, incl);
+                }
+                V ex = shfl_up(incl, 1);
+                if (lg == 0) ex = O::id();
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) a[k] = O::comb(ex, a[k]);
+            }
+            if (ok) {
+                Vec16<T> o;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) o.e[k] = O::val(a[k]);
+                *reinterpret_cast<int4 *>(out + v * VEC) = *reinterpret_cast<const int4 *>(&o);
+                if (out_idx)
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) out_idx[v * VEC + k] = O::idx(a[k]);
+            }
+        }
+    }
+    // ragged tail (L < VEC and n not a multiple of VEC): whole segments, one per thread
+    const int64_t t0 = nvec * VEC;
+    for (int64_t sgi = t0 / L + gid0; sgi * L < n; sgi += stride) {
+        V acc = O::id();
+        for (int j = 0; j < L; ++j) {
+            acc = j == 0 ? O::lift(x[sgi * L], 0) : O::fold(acc, x[sgi * L + j], j);
+            out[sgi * L + j] = O::val(acc);
+            if (out_idx) out_idx[sgi * L + j] = O::idx(acc);
+        }
+    }
+}
+
+// KS0 for rows that span 2..8 warps of a 256-thread CTA (32 * VEC < L <= 256 * VEC, L = 2^j):
+// a CTA takes U chunks of 256 consecutive vectors (each chunk = 256 * VEC / L whole
+// segments); every lane scans its vector in registers, every warp scans its lane totals
+// with shuffles, and the warps of a segment combine their totals through shared memory
+// (one barrier per U chunks).  No look-back, no flags: one read, one write per element.
+template <int OP, typename T, int U>
+__global__ void __launch_bounds__(256)
+segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    __shared__ V wt[U][8];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int WS = L / (32 * VEC);          // warps per segment (2, 4 or 8)
+    const int wr = warp & (WS - 1);         // rank of this warp within its segment
+    const int64_t nvec = n / VEC;  // whole segments are whole warps: a partial last chunk ends on a warp boundary
+    const int64_t nchunk = (nvec + 255) / 256;
+    for (int64_t c0 = (int64_t)blockIdx.x * U; c0 < nchunk; c0 += (int64_t)gridDim.x * U) {
+        int4 r[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if ((c0 + u) * 256 + threadIdx.x < nvec) r[u] = ldg16(x + ((c0 + u) * 256 + threadIdx.x) * VEC);
+        V a[U][VEC], ex[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const Vec16<T> e = as_vec<T>(r[u]);
+            const int j0 = (wr * 32 + lane) * VEC;  // segment-local index of the first element
+#pragma unroll
+            for (int k = 0; k < VEC; ++k)
+                a[u][k] = k == 0 ? O::lift(e.e[0], j0) : O::fold(a[u][k - 1], e.e[k], j0 + k);
+            V incl = a[u][VEC - 1];
+#pragma unroll
+            for (int dd = 1; dd < 32; dd <<= 1) {
+                const V y = shfl_up(incl, dd);
+                if (lane >= dd) incl = O::comb(y, incl);
+            }
+            ex[u] = shfl_up(incl, 1);
+            if (lane == 0) ex[u] = O::id();
+            if (lane == 31) wt[u][warp] = incl;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            V p = O::id();
+            for (int q = warp - wr; q < warp; ++q) p = O::comb(p, wt[u][q]);
+            ex[u] = O::comb(p, ex[u]);
+        }
+        __syncthreads();  // wt is reused by the next chunks
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = (c0 + u) * 256 + threadIdx.x;
+            if (v >= nvec) break;
+            Vec16<T> o;
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) {
+                const V z = O::comb(ex[u], a[u][k]);
+                o.e[k] = O::val(z);
+                if (out_idx) out_idx[v * VEC + k] = O::idx(z);
+            }
+            *reinterpret_cast<int4 *>(out + v * VEC) = *reinterpret_cast<const int4 *>(&o);
+        }
+    }
+}
+
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1522,6 +1664,26 @@ template <int OP, typename T> struct ScanRun {
             return FS_ERR_UNSUPPORTED;
         }
         if (seg) {
+            constexpr int64_t VEC = 16 / sizeof(T);
+            if (al && !carry && map->ibase == 0 && L >= 1 && L <= 32 * VEC && (L & (L - 1)) == 0) {
+                auto kv = segscan_vec_kernel<OP, T, 4>;
+                const int64_t nvec = n / VEC;
+                int64_t grid = ceil_div(nvec > 0 ? nvec : 1, 256 * 4);
+                const int64_t cap = resident_blocks((const void *)kv, 256);
+                grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
+                const int G = L > VEC ? (int)(L / VEC) : 1;
+                kv<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, G, (T *)out, out_idx);
+                return launch_status();
+            }
+            if (al && !carry && map->ibase == 0 && L > 32 * VEC && L <= 256 * VEC && (L & (L - 1)) == 0) {
+                auto kb = segscan_blk_kernel<OP, T, 2>;
+                const int64_t nchunk = ceil_div(n / VEC, 256);
+                int64_t grid = ceil_div(nchunk > 0 ? nchunk : 1, 2);
+                const int64_t cap = resident_blocks((const void *)kb, 256);
+                grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
+                kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
+                return launch_status();
+            }
             if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
             return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
         }

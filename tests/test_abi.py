@@ -197,7 +197,9 @@ def test_workspace_queries_and_regimes(fs):
     assert r(1 << 13, 1 << 15) == 2
     assert r(4, 1 << 26) == 3 and r(1, 1 << 28) == 3
     assert r(64, 64, layout="col") == 4
-    assert r(64, 64, scan=True) == 5
+    assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 5
+    assert r(1 << 10, 2048, scan=True) == 5
+    assert r(1 << 20, 512, scan=True, dtype=torch.int64) == 7 and r(1 << 20, 1024, scan=True, dtype=torch.int64) == 5
     assert r(0, 64) == 6 and r(64, 0) == 6
     assert r(64, 64, dtype=torch.int64, op="argmin") == 0
     fs.force_seg_regime(2)

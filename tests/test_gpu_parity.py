@@ -335,6 +335,26 @@ def test_seg_scan(fs, nseg, seglen, layout):
         assert_reduced(got, want, op, asum, f"segscan {layout} {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("seglen", [1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024])
+@pytest.mark.parametrize("nseg", [1, 3, 1001, 7_001])
+def test_seg_scan_short_pow2(fs, nseg, seglen):
+    """KS0 (regime 7): power-of-two rows by in-register + shuffle scans (one warp) and a
+    shared-memory combine across warps (256..1024 f32, 128..512 8-byte); every op and
+    dtype (8-byte types at 1024 go to the look-back scan), ragged vector tails for
+    L < 4, argmin ties, int wrap-around."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int32, "max"), (np.int64, "add"), (np.int64, "argmin"), (np.float32, "max")):
+        x = workloads.mixed(nseg * seglen, nseg + seglen, dt)
+        if op == "argmin" and x.size > 8:
+            x[::5] = x.min()  # ties inside segments: the first index must win
+        if dt == np.int32 and op == "add":
+            x = workloads.full_range(x.size, seglen, np.int32)
+        got = fs.seg_scan(cu(x), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan short {nseg}x{seglen} {dt.__name__} {op}")
+
+
 def test_seg_scan_misaligned(fs):
     x = workloads.mixed(50 * 999, 4, np.int64)
     got = fs.seg_scan(cu(x, 1), 50, 999, "add")
