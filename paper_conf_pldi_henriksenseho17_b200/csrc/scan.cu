@@ -1111,10 +1111,11 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
     extern __shared__ __align__(128) unsigned char sbuf[];
     unsigned char *ringA = sbuf, *ringC = sbuf + STA * TB;
     __shared__ uint64_t fullA[STA], emptyA[STA], fullC[STC], doneC[STC];
-    __shared__ volatile int s_c_slab;  // slab (local index) group C is working on
+    __shared__ int s_c_slab;  // slab (local index) group C is working on (shared-memory atomics: a
+                              // monotone progress flag read by the producer, no ordering needed)
     __shared__ V s_redA[NWA];
     __shared__ S s_wtot[2][NWC], s_lb_val[NWC];
-    __shared__ int s_lb_min[NWC];
+    __shared__ __align__(16) int s_lb_min[NWC];  // 16-byte aligned: its vector loads stay inside it
     const int G = gridDim.x, b = blockIdx.x;
     const int64_t nslabs = (ntiles + tps - 1) / tps;
     const int my_slabs = (int)((nslabs - b + G - 1) / G);
@@ -1148,7 +1149,7 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
             // A: a slot is released when all of group A has consumed its tile
             while (a_rel < a_iss && mbar_test(&emptyA[a_rel % STA], (unsigned)(a_rel / STA) & 1u)) ++a_rel;
             // A: issue while a slot is free and A stays within DA slabs of C
-            while (a_iss < my_tiles && a_iss < a_rel + STA && a_iss / tps - FS_SCANW_DA <= s_c_slab) {
+            while (a_iss < my_tiles && a_iss < a_rel + STA && a_iss / tps - FS_SCANW_DA <= atomicAdd(&s_c_slab, 0)) {
                 const int64_t t = tile_at(a_iss);
                 if (full_tile(t)) {
                     const int s = a_iss % STA;
@@ -1267,7 +1268,7 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
     int j = 0;
     for (int m = 0; m < my_slabs; ++m) {
         const int64_t slab = slab_of(m);
-        if (ct == 0) s_c_slab = m;
+        if (ct == 0) atomicExch(&s_c_slab, m);
         S exc = SO::id();
         if (slab == 0) {
             if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};

@@ -42,5 +42,18 @@ fs.stream_red(cu(pts), cu(mem), 32)
 fs.stream_red(cu(workloads.mixed((3000, 100), 4, np.float32)), cu(workloads.ints(3000, 5, 0, 70)), 70)
 fs.transpose_2d(cu(workloads.mixed((333, 517), 6, np.float32)))
 fs.transpose_2d(cu(workloads.mixed((256, 128), 7, np.int64)))
+# seg_scan KS0 (power-of-two rows: one warp, several warps, ragged tail)
+for nseg, L in ((1001, 2), (999, 16), (300, 128), (101, 512), (37, 1024)):
+    fs.seg_scan(x[: nseg * L], nseg, L, "add")
+    fs.seg_scan(x[: nseg * L], nseg, L, "argmin")
+    fs.seg_scan(xi[: nseg * L], nseg, L, "min")
+# NEXT-2 nn_knn (cooperative launch, grid barrier) and NEXT-1 kmeans_step
+lat2, lng2, q2 = workloads.c2_nn(base=30_000, reps=3)
+fs.nn_knn(cu(lat2), cu(lng2), q2, 100)
+fs.nn_knn(cu(lat2[:777]), cu(lng2[:777]), q2, 1000)
+pts, _ = workloads.c3_kmeans(n=20_011, d=34, k=32)
+fs.kmeans_step(cu(pts), cu(pts[:32].copy()), prev=cu(workloads.ints(20_011, 3, 0, 32)))
+pts, _ = workloads.c3_kmeans(n=5_003, d=7, k=5)
+fs.kmeans_step(cu(pts), cu(pts[:5].copy()))
 torch.cuda.synchronize()
 print("sanitize cases done")
