@@ -1876,8 +1876,74 @@ colscan_kernel(const T *__restrict__ x, int64_t m, int64_t w, int64_t WV, int64_
     }
 }
 
+// ---------------------------------------------------------------- narrow column-major seg_scan
+// Few columns (a row of w elements is WV <= 8 16-byte vectors, WV | 32): a WARP owns a block
+// of rows and its lanes read 32 / WV consecutive rows at a time (lane l: row l / WV, vector
+// column l % WV), so every warp load is one contiguous 512-byte run.  The per-thread
+// (vector-column, row-block) units of the generic kernels above would give every lane its
+// own row block and thrash L1 when rows are this short.  Partial: fold, then combine the
+// row-lanes of each column with xor shuffles.  Scan: per 32/WV-row step, an inclusive shuffle
+// scan down the row-lanes of each column plus the running carry.
+template <int OP, typename T, bool CARRY, bool SCAN>
+__global__ void __launch_bounds__(kColScanThreads)
+colscan_narrow_kernel(const T *__restrict__ x, int64_t m, int64_t w, int WV, int64_t Y, int64_t rpu,
+                      typename Op<OP, T>::V *parts, T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    const int lane = threadIdx.x & 31;
+    const int64_t y = ((int64_t)blockIdx.x * kColScanThreads + threadIdx.x) >> 5;  // warp = unit
+    if (y >= Y) return;
+    const int cv = lane % WV, ro = lane / WV, RPW = 32 / WV;
+    const int64_t r0 = y * rpu, r1 = r0 + rpu < m ? r0 + rpu : m;
+    V acc[VEC];
+#pragma unroll
+    for (int k = 0; k < VEC; ++k) acc[k] = CARRY ? parts[y * w + cv * VEC + k] : O::id();
+    for (int64_t rb = r0; rb < r1; rb += RPW) {
+        const int64_t r = rb + ro;
+        const bool ok = r < r1;
+        Vec16<T> e;
+        if (ok) e = as_vec<T>(ldg16(x + r * w + cv * VEC));
+        if (!SCAN) {
+            if (ok)
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) acc[k] = O::comb(acc[k], O::lift(e.e[k], r));
+            continue;
+        }
+        V v[VEC];
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) v[k] = ok ? O::lift(e.e[k], r) : O::id();
+#pragma unroll 1
+        for (int dd = 1; dd < RPW; dd <<= 1) {
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) {
+                const V o = shfl_up(v[k], dd * WV);
+                if (ro >= dd) v[k] = O::comb(o, v[k]);
+            }
+        }
+        Vec16<T> o;
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) {
+            const V z = O::comb(acc[k], v[k]);
+            o.e[k] = O::val(z);
+            if (ok && OP == kArgmin) out_idx[r * w + cv * VEC + k] = O::idx(z);
+            acc[k] = shfl_idx(z, (RPW - 1) * WV + cv);  // carry = the step's last row of this column
+        }
+        if (ok) *reinterpret_cast<int4 *>(out + r * w + cv * VEC) = *reinterpret_cast<const int4 *>(&o);
+    }
+    if (!SCAN) {
+        for (int dd = WV; dd < 32; dd <<= 1)
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) acc[k] = O::comb(acc[k], shfl_xor(acc[k], dd));
+        if (ro == 0)
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) parts[y * w + cv * VEC + k] = acc[k];
+    }
+}
+
 struct ColScanPlan {
     int vec;
+    bool narrow;  // colscan_narrow_kernel: a warp per row block
     int64_t WV, Y, rpu;
 };
 static ColScanPlan colscan_plan(int dt, int64_t m, int64_t w, bool aligned) {
@@ -1885,6 +1951,17 @@ static ColScanPlan colscan_plan(int dt, int64_t m, int64_t w, bool aligned) {
     const int V = 16 / (int)dtype_size(dt);
     p.vec = (aligned && w % V == 0) ? V : 1;
     p.WV = ceil_div(w, p.vec);
+    p.narrow = p.vec > 1 && p.WV <= 8 && (32 % p.WV) == 0 && m >= 4096;
+    if (p.narrow) {  // warps (units) of 32 / WV-row steps
+        int64_t Y = (int64_t)sm_count() * (2048 / 32);
+        const int64_t by_rows = m / 256;
+        if (Y > by_rows) Y = by_rows;
+        if (Y < 1) Y = 1;
+        const int64_t step = 32 / p.WV;
+        p.rpu = ceil_div(ceil_div(m, Y), step) * step;
+        p.Y = ceil_div(m, p.rpu);
+        return p;
+    }
     const int64_t threads = (int64_t)sm_count() * 2048;
     int64_t Y = ceil_div(threads, p.WV);
     const int64_t by_rows = m / 16;
@@ -1901,6 +1978,26 @@ template <int OP, typename T> struct ColScanRun {
                         cudaStream_t st) {
         using V = typename Op<OP, T>::V;
         V *parts = (V *)((char *)ws + kWsHeader);
+        if (p.narrow) {
+            const unsigned gn = (unsigned)ceil_div(p.Y * 32, kColScanThreads);
+            const int wv = (int)p.WV;
+            if (p.Y == 1) {
+                colscan_narrow_kernel<OP, T, false, true><<<gn, kColScanThreads, 0, st>>>(x, m, w, wv, 1, p.rpu, parts,
+                                                                                         out, out_idx);
+                return launch_status();
+            }
+            colscan_narrow_kernel<OP, T, false, false><<<gn, kColScanThreads, 0, st>>>(x, m, w, wv, p.Y, p.rpu, parts,
+                                                                                      out, out_idx);
+            if (p.Y >= 256) {
+                colscan_carry_block_kernel<OP, T><<<(unsigned)w, 256, 0, st>>>(parts, w, p.Y);
+            } else {
+                int64_t g2 = ceil_div(w, 128);
+                colscan_carry_kernel<OP, T><<<(unsigned)(g2 > 4096 ? 4096 : g2), 128, 0, st>>>(parts, w, p.Y);
+            }
+            colscan_narrow_kernel<OP, T, true, true><<<gn, kColScanThreads, 0, st>>>(x, m, w, wv, p.Y, p.rpu, parts,
+                                                                                    out, out_idx);
+            return launch_status(3);
+        }
         const int64_t units = p.WV * p.Y;
         const unsigned grid = (unsigned)ceil_div(units, kColScanThreads);
         if (p.Y == 1) {

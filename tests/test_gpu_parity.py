@@ -355,6 +355,24 @@ def test_seg_scan_short_pow2(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan short {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("nseg,seglen", [(4, 70_001), (8, 4096), (16, 100_003), (32, 9_999), (2, 300_007),
+                                         (4, 2_000_000)])
+def test_seg_scan_col_narrow(fs, nseg, seglen):
+    """Column-major seg_scan with few columns (rows of <= 8 16-byte vectors): the warp-per-
+    row-block kernels (partial, carry, scan); ragged row blocks; argmin ties; 8-byte types."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int64, "add"), (np.int32, "max")):
+        if np.dtype(dt).itemsize == 8 and nseg > 16:
+            continue
+        x = workloads.mixed(nseg * seglen, nseg * 7 + seglen, dt)
+        if op == "argmin":
+            x[::3] = x.min()
+        got = fs.seg_scan(cu(x), nseg, seglen, op, layout="col")
+        want = oracle.seg_scan(x, nseg, seglen, op, "col")
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", "col") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan col narrow {nseg}x{seglen} {dt.__name__} {op}")
+
+
 def test_seg_scan_misaligned(fs):
     x = workloads.mixed(50 * 999, 4, np.int64)
     got = fs.seg_scan(cu(x, 1), 50, 999, "add")
