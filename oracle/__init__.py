@@ -61,8 +61,9 @@ def _L():
         lib.orc_transpose.argtypes = [L, P, L, L, P]
         lib.orc_nn_knn.argtypes = [P, P, L, ctypes.c_float, ctypes.c_float, L, P, P, P, P]
         lib.orc_kmeans_step.argtypes = [P, L, L, P, L, P, P, P, P, P, P]
+        lib.orc_seg_map_reduce.argtypes = [I, I, P, L, L, L, ctypes.c_float, P, P, P]
         for f in ("orc_reduce", "orc_scan", "orc_nn_dist", "orc_vreduce", "orc_seg_reduce",
-                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn", "orc_kmeans_step"):
+                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn", "orc_kmeans_step", "orc_seg_map_reduce"):
             getattr(lib, f).restype = I
         _lib = lib
     return _lib
@@ -186,6 +187,21 @@ def seg_reduce(x, nseg, seglen, op="add", layout="row"):
     _check(_L().orc_seg_reduce(OPS[op], _DT[x.dtype], _p(x), nseg, seglen, LAYOUTS[layout],
                                _p(out), _p(idx)), "seg_reduce")
     return (out, idx) if op == "argmin" else out
+
+
+def seg_map_reduce(x, nseg, seglen, c, op="add"):
+    """NEXT-4, L247-252: map (\\row -> (map (+c) row, reduce op row)) over the row-major
+    [nseg][seglen] x.  Returns (mapped [nseg*seglen] of x's dtype, reduced [nseg]
+    (f64 for f32 add) [, argmin index])."""
+    x = _arr(x).reshape(-1)
+    assert x.size == nseg * seglen
+    mapped = np.zeros(x.size, x.dtype)
+    out = np.zeros(nseg, _out_dtype(op, x.dtype))
+    idx = np.full(nseg, -7, np.int64)
+    ci = int(c) if x.dtype.kind == "i" else 0
+    _check(_L().orc_seg_map_reduce(OPS[op], _DT[x.dtype], _p(x), nseg, seglen, ci, float(c), _p(mapped), _p(out),
+                                   _p(idx)), "seg_map_reduce")
+    return (mapped, out, idx) if op == "argmin" else (mapped, out)
 
 
 def seg_scan(x, nseg, seglen, op="add", layout="row"):

@@ -334,3 +334,26 @@ int orc_kmeans_step(const float *x, int64_t n, int64_t d, const float *cen, int6
     if (delta) *delta = prev ? changed : 0;
     return 0;
 }
+
+/* NEXT-4, the horizontally fused row nest of L247-252:
+ *     map (\row -> (map (\x -> x + c) row, reduce (+) 0 row)) matrix
+ * generalised to the operator table for the reduce: for every row s of the
+ * row-major [nseg][seglen] x,
+ *     out_map[s][j] = x[s][j] + c    (i32/i64: wraps, R1; f32: one f32 add)
+ *     out_red[s]    = reduce op 0(op) x[s]   (over the ORIGINAL row, as in L250)
+ * c is ci for integer types and cf for f32.  Straight loops, no fusion. */
+int orc_seg_map_reduce(int op, int dt, const void *x, int64_t nseg, int64_t seglen, int64_t ci, float cf,
+                       void *out_map, void *out_red, int64_t *out_idx) {
+    if (!valid(op, dt) || nseg < 0 || seglen < 0) return 1;
+    if (nseg > 0 && seglen > 0 && (!x || !out_map)) return 1;
+    for (int64_t e = 0; e < nseg * seglen; ++e) {
+        if (dt == ORC_F32) {
+            ((float *)out_map)[e] = ((const float *)x)[e] + cf;
+        } else if (dt == ORC_I32) {
+            ((int32_t *)out_map)[e] = (int32_t)((uint32_t)((const int32_t *)x)[e] + (uint32_t)ci);
+        } else {
+            ((int64_t *)out_map)[e] = (int64_t)((uint64_t)((const int64_t *)x)[e] + (uint64_t)ci);
+        }
+    }
+    return orc_seg_reduce(op, dt, x, nseg, seglen, ORC_ROW_MAJOR, out_red, out_idx);
+}

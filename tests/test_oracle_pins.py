@@ -293,6 +293,32 @@ def test_kmeans_step_closed_forms():
     np.testing.assert_allclose(s_sr, s_k, rtol=1e-12)
 
 
+def test_golden_l247_map_reduce():
+    g = gold("l247_map_reduce.json")
+    x = np.array(g["matrix"], np.float32)
+    mapped, sums = oracle.seg_map_reduce(x, 2, 3, g["c"])
+    assert mapped.reshape(2, 3).tolist() == g["mapped"] and sums.tolist() == g["sums"]
+
+
+@pytest.mark.parametrize("dt", DTYPES)
+def test_seg_map_reduce_against_numpy(dt):
+    """The mapped output is numpy's x + c (f32: the same single rounding; ints: wrap-around);
+    the reduced output is seg_reduce of the ORIGINAL rows (pinned above)."""
+    x = workloads.full_range((37, 129), 11, dt) if np.dtype(dt).kind == "i" else workloads.mixed((37, 129), 11, dt)
+    c = 7 if np.dtype(dt).kind == "i" else 0.37
+    for op in OPS:
+        r = oracle.seg_map_reduce(x, 37, 129, c, op)
+        want_map = (x.reshape(-1) + np.array(c, dt)).astype(dt) if np.dtype(dt).kind == "f" else \
+            (x.reshape(-1).astype(np.int64 if dt == np.int32 else np.uint64) + c).astype(dt)
+        np.testing.assert_array_equal(r[0], want_map)
+        want_red = oracle.seg_reduce(x, 37, 129, op)
+        if op == "argmin":
+            np.testing.assert_array_equal(r[1], want_red[0])
+            np.testing.assert_array_equal(r[2], want_red[1])
+        else:
+            np.testing.assert_array_equal(r[1], want_red)
+
+
 def test_invalid_key_is_rejected():
     with pytest.raises(ValueError):
         oracle.stream_red(np.ones((3, 2), np.float32), np.array([0, 5, 1]), 3)
