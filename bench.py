@@ -248,6 +248,19 @@ def time_next_rows(fs, W, dev, K, peak):
                                       "tflops_tf32": round(flops / (avg * 1e-3) / 1e12, 1),
                                       "note": "fused assignment (mma.sync TF32 + exact near-tie re-evaluation) + "
                                               "stream_red + new centres + delta; membership bit-exact vs f32 oracle"}
+    # NEXT-4: the L247-252 row nest (map (+1.0) row, reduce (+) row) over the C5 matrix
+    # [2^14][2^14] f32 and over C4 rows [2^18][1024]: one read, two outputs
+    for name, xm, nseg, L in (("seg_map_reduce_2^14x2^14", W["tmat"], W["t"], W["t"]),
+                              ("seg_map_reduce_2^18x1024", W["x"], W["n"] // 1024, 1024)):
+        om = torch.empty_like(xm)
+        orow = torch.empty(nseg, dtype=torch.float32, device=dev)
+        avg, mn = timed(lambda: fs.seg_map_reduce(xm, nseg, L, 1.0, "add", out_map=om, out=orow))
+        b = 8 * nseg * L + 4 * nseg
+        rows[name] = {"ms": round(avg, 4), "ms_min": round(mn, 4), "GB_s": round(b / (avg * 1e-3) / GB, 1),
+                      "elements_per_s": float(f"{nseg * L / (avg * 1e-3):.4g}"), "bytes": b,
+                      "frac_of_peak": round(b / (avg * 1e-3) / GB / peak, 4),
+                      "note": "x read once; x + 1.0 written and every row summed"}
+        del om
     return rows
 
 

@@ -234,6 +234,20 @@ fs_status fs_kmeans_step(const float *points, int64_t n, int64_t d, const float 
                          const int32_t *prev, int32_t *membership, float *sums, int32_t *counts,
                          float *new_centres, int64_t *delta, void *ws, size_t ws_bytes, void *stream);
 
+/* ---------------------------------------------------------------- NEXT-4: seg_map_reduce */
+/* The horizontally fused row nest of L247-252,
+ *     map (\row -> (map (\x -> x + c) row, reduce (+) 0 row)) matrix,
+ * with the reduce from the operator table: for every row s of the row-major
+ * [nseg][seglen] array `in`, in ONE read of the row,
+ *   out_map[s][j] = in[s][j] + c          (I32/I64: c = c_int, wraps; F32: c = c_f32)
+ *   out[s]        = reduce op 0(op) in[s] (the ORIGINAL row; ARGMIN: out_idx[s] is the
+ *                                           row-local index, -1 for an empty row)
+ *   op.op in {ADD, MIN, MAX, ARGMIN}; out_map has in's shape; no output may overlap an
+ *   input or another output (FS_ERR_ALIAS). */
+fs_status fs_seg_map_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, size_t *bytes);
+fs_status fs_seg_map_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int64_t c_int, float c_f32,
+                            void *out_map, void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
+
 /* ---------------------------------------------------------------- utilities */
 /* Synchronises `stream`, reads and clears the device error word of `ws`.
  * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */

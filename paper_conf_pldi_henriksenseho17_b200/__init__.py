@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "kmeans_step", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "kmeans_step", "seg_map_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -73,6 +73,8 @@ _SIG = {
     "fs_nn_knn": [_P, _P, _L, ctypes.c_float, ctypes.c_float, _L, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_kmeans_step_workspace": [_L, _L, _L, _SZ],
     "fs_kmeans_step": [_P, _L, _L, _P, _L, _P, _P, _P, _P, _P, _P, _P, ctypes.c_size_t, _P],
+    "fs_seg_map_reduce_workspace": [fs_opdesc, _L, _L, _SZ],
+    "fs_seg_map_reduce": [fs_opdesc, _P, _L, _L, _L, ctypes.c_float, _P, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
@@ -285,6 +287,27 @@ def kmeans_step(points, centres, prev=None, membership=None, sums=None, counts=N
                             _ptr(counts), _ptr(new_centres), _ptr(delta), ctypes.c_void_p(ws.data_ptr()), ws.numel(),
                             _stream(dev)), "fs_kmeans_step")
     return membership, sums, counts, new_centres, delta
+
+
+def seg_map_reduce(x, nseg: int, seglen: int, c, op: str = "add", out_map=None, out=None, out_idx=None):
+    """NEXT-4, L247-252: for every row of the row-major [nseg][seglen] x, in one read:
+    (map (+c) row, reduce op row).  Returns (mapped [like x], reduced [nseg] [, idx])."""
+    x = _dev(x, "x")
+    dt = _dt(x)
+    if x.numel() != nseg * seglen:
+        raise ValueError("seg_map_reduce: x must hold nseg * seglen elements")
+    o = _op(op, dt)
+    if out_map is None:
+        out_map = torch.empty_like(x)
+    if out is None:
+        out = torch.empty(nseg, dtype=x.dtype, device=x.device)
+    if op == "argmin" and out_idx is None:
+        out_idx = torch.empty(nseg, dtype=torch.int64, device=x.device)
+    ci = int(c) if dt != FS_F32 else 0
+    ws = workspace(_query(_lib.fs_seg_map_reduce_workspace, o, nseg, seglen), x.device)
+    _ok(_lib.fs_seg_map_reduce(o, _ptr(x), nseg, seglen, ci, float(c), _ptr(out_map), _ptr(out), _ptr(out_idx),
+                               ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(x.device)), "fs_seg_map_reduce")
+    return (out_map, out, out_idx) if op == "argmin" else (out_map, out)
 
 
 def stream_red(vals, keys, k: int, sums=None, counts=None, with_counts: bool = True):

@@ -421,6 +421,37 @@ fs_status fs_kmeans_step(const float *points, int64_t n, int64_t d, const float 
     return kmeans_run(points, n, d, centres, k, prev, membership, sums, counts, new_centres, delta, ws, S(stream));
 }
 
+// ------------------------------------------------------------ NEXT-4: seg_map_reduce
+fs_status fs_seg_map_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    FS_TRY(check_op(op, false));
+    if (nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen) || mul_overflows(nseg * seglen, 8)) return FS_ERR_SIZE;
+    *bytes = seg_map_reduce_ws(op.op, op.dtype, nseg, seglen);
+    return FS_OK;
+}
+
+fs_status fs_seg_map_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int64_t c_int, float c_f32,
+                            void *out_map, void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream) {
+    size_t need = 0;
+    FS_TRY(fs_seg_map_reduce_workspace(op, nseg, seglen, &need));
+    if (nseg == 0) return FS_OK;
+    if (!out || (seglen > 0 && (!in || !out_map)) || (op.op == FS_ARGMIN && !out_idx)) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(op.dtype), nb = nseg * seglen * es;
+    if ((in && !aligned_to(in, es)) || (out_map && !aligned_to(out_map, es)) || !aligned_to(out, es) ||
+        (out_idx && !aligned_to(out_idx, 8)))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t ob = nseg * es, ib8 = out_idx ? nseg * 8 : 0;
+    if (overlaps(out_map, nb, in, nb) || overlaps(out, ob, in, nb) || overlaps(out, ob, out_map, nb) ||
+        (out_idx && (overlaps(out_idx, ib8, in, nb) || overlaps(out_idx, ib8, out_map, nb) ||
+                     overlaps(out_idx, ib8, out, ob))))
+        return FS_ERR_ALIAS;
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    if (seglen == 0) return fill_neutral_run(op.op, op.dtype, nseg, out, op.op == FS_ARGMIN ? out_idx : nullptr,
+                                             S(stream));
+    return seg_map_reduce_run(op.op, op.dtype, in, nseg, seglen, c_int, c_f32, out_map, out,
+                              op.op == FS_ARGMIN ? out_idx : nullptr, ws, S(stream));
+}
+
 // ------------------------------------------------------------ utilities
 fs_status fs_check_device_error(void *ws, void *stream) {
     if (!ws) return FS_ERR_NULL;

@@ -89,6 +89,10 @@ size_t kmeans_ws(int64_t n, int64_t d, int64_t k);
 fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, int64_t k, const int32_t *prev,
                      int32_t *membership, float *sums, int32_t *counts, float *new_cen, int64_t *delta, void *ws,
                      cudaStream_t st);
+// seg_map_reduce.cu (NEXT-4)
+size_t seg_map_reduce_ws(int op, int dt, int64_t nseg, int64_t L);
+fs_status seg_map_reduce_run(int op, int dt, const void *in, int64_t nseg, int64_t L, int64_t ci, float cf, void *ymap,
+                             void *out, int64_t *out_idx, void *ws, cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 

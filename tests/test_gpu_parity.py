@@ -150,6 +150,38 @@ def test_kmeans_step_c3_kdd_and_ties(fs):
         _km_check(fs, small, cen, None, f"n={n}")
 
 
+# ------------------------------------------------------------------ NEXT-4: seg_map_reduce
+@pytest.mark.parametrize("nseg,seglen", [(1, 1), (1000, 1), (777, 3), (4096, 4), (300, 32), (1000, 33), (64, 128),
+                                         (50, 1000), (9, 4097), (3, 65537), (2, 1_000_003), (0, 5), (7, 0)])
+def test_seg_map_reduce(fs, nseg, seglen):
+    """L247-252 fused row nest: x + c written and each row reduced in one read; every op,
+    all dtypes, short power-of-two rows (shuffle groups), warp rows, rows cut into pieces."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int32, "max"), (np.int64, "argmin")):
+        x = workloads.mixed(nseg * seglen, nseg * 5 + seglen, dt)
+        if op == "argmin" and x.size > 10:
+            x[::7] = x.min()
+        c = 3 if np.dtype(dt).kind == "i" else 1.0
+        got = fs.seg_map_reduce(cu(x), nseg, seglen, c, op)
+        want = oracle.seg_map_reduce(x, nseg, seglen, c, op)
+        np.testing.assert_array_equal(host(got[0]).reshape(-1), want[0])  # the map: exact
+        rest_got = (got[1], got[2]) if op == "argmin" else got[1]
+        rest_want = (want[1], want[2]) if op == "argmin" else want[1]
+        asum = oracle.seg_reduce(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(rest_got, rest_want, op, asum, f"seg_map_reduce {nseg}x{seglen} {dt.__name__} {op}")
+
+
+def test_seg_map_reduce_misaligned(fs):
+    """Input and output with different 16-byte phases (scalar map stores) and odd offsets."""
+    x = workloads.mixed(37 * 1001, 9, np.float32)
+    xin = cu(x, 1)
+    om = torch.empty(x.size + 2, dtype=torch.float32, device="cuda")[2:]
+    got = fs.seg_map_reduce(xin, 37, 1001, 0.5, "add", out_map=om)
+    want = oracle.seg_map_reduce(x, 37, 1001, 0.5, "add")
+    np.testing.assert_array_equal(host(got[0]), want[0])
+    assert_reduced(got[1], want[1], "add", oracle.seg_reduce(np.abs(x), 37, 1001, "add"), "misaligned")
+
+
 # ------------------------------------------------------------------ NEXT-2: nn_knn
 def _knn_check(fs, lat, lng, q, kk, off=0):
     d, i = fs.nn_knn(cu(lat, off), cu(lng, off), q, kk)
