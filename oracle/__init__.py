@@ -62,8 +62,9 @@ def _L():
         lib.orc_nn_knn.argtypes = [P, P, L, ctypes.c_float, ctypes.c_float, L, P, P, P, P]
         lib.orc_kmeans_step.argtypes = [P, L, L, P, L, P, P, P, P, P, P]
         lib.orc_seg_map_reduce.argtypes = [I, I, P, L, L, L, ctypes.c_float, P, P, P]
+        lib.orc_scan_reduce.argtypes = [I, I, I, P, L, P]
         for f in ("orc_reduce", "orc_scan", "orc_nn_dist", "orc_vreduce", "orc_seg_reduce",
-                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn", "orc_kmeans_step", "orc_seg_map_reduce"):
+                  "orc_seg_scan", "orc_stream_red", "orc_transpose", "orc_nn_knn", "orc_kmeans_step", "orc_seg_map_reduce", "orc_scan_reduce"):
             getattr(lib, f).restype = I
         _lib = lib
     return _lib
@@ -202,6 +203,15 @@ def seg_map_reduce(x, nseg, seglen, c, op="add"):
     _check(_L().orc_seg_map_reduce(OPS[op], _DT[x.dtype], _p(x), nseg, seglen, ci, float(c), _p(mapped), _p(out),
                                    _p(idx)), "seg_map_reduce")
     return (mapped, out, idx) if op == "argmin" else (mapped, out)
+
+
+def scan_reduce(x, scan_op="add", red_op="add"):
+    """NEXT-3, Fig 10a: reduce red_op (scan scan_op x), the scan materialised (unfused).
+    f32 results in f64."""
+    x = _arr(x).reshape(-1)
+    out = np.zeros(1, np.float64 if x.dtype == np.float32 else x.dtype)
+    _check(_L().orc_scan_reduce(OPS[scan_op], OPS[red_op], _DT[x.dtype], _p(x), x.size, _p(out)), "scan_reduce")
+    return out[0]
 
 
 def seg_scan(x, nseg, seglen, op="add", layout="row"):

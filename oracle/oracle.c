@@ -357,3 +357,24 @@ int orc_seg_map_reduce(int op, int dt, const void *x, int64_t nseg, int64_t segl
     }
     return orc_seg_reduce(op, dt, x, nseg, seglen, ORC_ROW_MAJOR, out_red, out_idx);
 }
+
+/* NEXT-3, Fig 10a (L1158-1170) with g = id: the scan is materialised and reduced,
+ *     y = scan (scan_op) x;   out = reduce (red_op) y
+ * exactly the unfused program (F5 and F4 fuse it into one stream_seq, F7; the
+ * library computes the fused form).  f32 in f64 (R2; the result is returned as a
+ * double), integers wrap (R1). */
+int orc_scan_reduce(int scan_op, int red_op, int dt, const void *x, int64_t n, void *out) {
+    if (!valid(scan_op, dt) || !valid(red_op, dt) || scan_op == ORC_ARGMIN || red_op == ORC_ARGMIN || n < 0 ||
+        !out || (n > 0 && !x))
+        return 1;
+    val_t s = neutral(scan_op, dt), r = neutral(red_op, dt);
+    for (int64_t i = 0; i < n; ++i) {
+        s = combine(scan_op, dt, s, load(dt, x, i, i));  /* y[i] */
+        val_t y = s;
+        y.idx = i;
+        r = combine(red_op, dt, r, y);
+    }
+    if (dt == ORC_F32) ((double *)out)[0] = r.f;  /* f64 for f32 (R2), whatever red_op */
+    else store(red_op, dt, out, 0, r, 0);
+    return 0;
+}

@@ -319,6 +319,30 @@ def test_seg_map_reduce_against_numpy(dt):
             np.testing.assert_array_equal(r[1], want_red)
 
 
+@pytest.mark.parametrize("dt", DTYPES)
+def test_scan_reduce_against_numpy_and_closed_forms(dt):
+    """Fig 10a: reduce (scan x) = numpy cumsum then sum / max / min (f64 for f32, wrapping
+    int64 arithmetic for ints); closed forms: sum of the prefix sums of ones = n(n+1)/2,
+    of iota = sum_i i(i+1)/2; max prefix sum of a +1/-1 walk = its running maximum."""
+    x = workloads.mixed(10_007, 21, dt)
+    wide = x.astype(np.float64) if dt == np.float32 else x.astype(np.int64)
+    cs = np.cumsum(wide)
+    def wrap(v):
+        return np.array(v).astype(np.int64).astype(dt) if dt != np.float32 else v
+    if dt == np.float32:  # numpy sums pairwise: same f64 value up to rounding order
+        assert abs(oracle.scan_reduce(x, "add", "add") - np.sum(cs)) <= 1e-12 * np.sum(np.abs(cs))
+    else:
+        assert oracle.scan_reduce(x, "add", "add") == wrap(np.sum(cs))
+    assert oracle.scan_reduce(x, "add", "max") == (cs.max() if dt == np.float32 else wrap(cs.max()))
+    assert oracle.scan_reduce(x, "add", "min") == (cs.min() if dt == np.float32 else wrap(cs.min()))
+    n = 1000
+    assert oracle.scan_reduce(np.ones(n, dt), "add", "add") == n * (n + 1) // 2
+    assert oracle.scan_reduce(np.arange(n, dtype=dt), "add", "add") == sum(i * (i + 1) // 2 for i in range(n))
+    walk = np.where(np.arange(n) % 3 == 0, -1, 1).astype(dt)
+    assert oracle.scan_reduce(walk, "add", "max") == np.cumsum(walk.astype(np.int64)).max()
+    assert oracle.scan_reduce(np.zeros(0, dt), "add", "add") == 0  # empty: the reduce's neutral
+
+
 def test_invalid_key_is_rejected():
     with pytest.raises(ValueError):
         oracle.stream_red(np.ones((3, 2), np.float32), np.array([0, 5, 1]), 3)
