@@ -248,6 +248,19 @@ def time_next_rows(fs, W, dev, K, peak):
                                       "tflops_tf32": round(flops / (avg * 1e-3) / 1e12, 1),
                                       "note": "fused assignment (mma.sync TF32 + exact near-tie re-evaluation) + "
                                               "stream_red + new centres + delta; membership bit-exact vs f32 oracle"}
+    # NEXT-3: Fig 10c's fused stream_seq, reduce (scan x) in one read (2^28 f32, C4), vs
+    # the unfused program (scanomap materialised, then redomap)
+    x, n = W["x"], W["n"]
+    o1 = torch.empty((), dtype=torch.float32, device=dev)
+    for red in ("add", "max"):
+        avg, mn = timed(lambda: fs.scan_reduce(x, red, out=o1))
+        avg_u, _ = timed(lambda: fs.redomap(fs.scanomap(x, "add", out=W["o_scan"]), red, out=o1))
+        b = 4 * n
+        rows[f"scan_reduce_{red}_2^28"] = {"ms": round(avg, 4), "ms_min": round(mn, 4),
+                                          "GB_s": round(b / (avg * 1e-3) / GB, 1),
+                                          "elements_per_s": float(f"{n / (avg * 1e-3):.4g}"), "bytes": b,
+                                          "frac_of_peak": round(b / (avg * 1e-3) / GB / peak, 4),
+                                          "vs_unfused_scan_then_reduce_ms": round(avg_u, 4)}
     # NEXT-4: the L247-252 row nest (map (+1.0) row, reduce (+) row) over the C5 matrix
     # [2^14][2^14] f32 and over C4 rows [2^18][1024]: one read, two outputs
     for name, xm, nseg, L in (("seg_map_reduce_2^14x2^14", W["tmat"], W["t"], W["t"]),

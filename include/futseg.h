@@ -248,6 +248,21 @@ fs_status fs_seg_map_reduce_workspace(fs_opdesc op, int64_t nseg, int64_t seglen
 fs_status fs_seg_map_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen, int64_t c_int, float c_f32,
                             void *out_map, void *out, int64_t *out_idx, void *ws, size_t ws_bytes, void *stream);
 
+/* ---------------------------------------------------------------- NEXT-3: scan_reduce */
+/* The stream_seq fusion of Fig 10 (L1158-1227; F4, F5, F7 of Fig 9):
+ *     out = reduce red (scan (+) 0 x)
+ * computed in ONE read without materialising the scan: chunks are summarised by the
+ * fused (associative, non-commutative) pair operator and combined in index order.
+ *   red in {FS_ADD (sum of the prefix sums), FS_MAX / FS_MIN (max / min prefix sum)};
+ *   the scan operator is FS_ADD (others: FS_ERR_UNSUPPORTED); dtype I32/I64 or F32
+ *   (reassociated; the cross-warp combine in f64).  out: 1 element of dtype; n = 0 gives
+ *   red's neutral element.  Integer FS_ADD is exact under wrap-around; integer
+ *   FS_MAX/FS_MIN are exact when no prefix sum overflows (precondition: the pair
+ *   operator max(M1, A1 + M2) needs monotone addition). */
+fs_status fs_scan_reduce_workspace(int32_t dtype, int64_t n, size_t *bytes);
+fs_status fs_scan_reduce(int32_t scan_op, int32_t red_op, int32_t dtype, const void *in, int64_t n, void *out,
+                         void *ws, size_t ws_bytes, void *stream);
+
 /* ---------------------------------------------------------------- utilities */
 /* Synchronises `stream`, reads and clears the device error word of `ws`.
  * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */

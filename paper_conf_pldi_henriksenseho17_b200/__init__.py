@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "kmeans_step", "seg_map_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "kmeans_step", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -75,6 +75,8 @@ _SIG = {
     "fs_kmeans_step": [_P, _L, _L, _P, _L, _P, _P, _P, _P, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_seg_map_reduce_workspace": [fs_opdesc, _L, _L, _SZ],
     "fs_seg_map_reduce": [fs_opdesc, _P, _L, _L, _L, ctypes.c_float, _P, _P, _P, _P, ctypes.c_size_t, _P],
+    "fs_scan_reduce_workspace": [_I, _L, _SZ],
+    "fs_scan_reduce": [_I, _I, _I, _P, _L, _P, _P, ctypes.c_size_t, _P],
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
@@ -308,6 +310,19 @@ def seg_map_reduce(x, nseg: int, seglen: int, c, op: str = "add", out_map=None, 
     _ok(_lib.fs_seg_map_reduce(o, _ptr(x), nseg, seglen, ci, float(c), _ptr(out_map), _ptr(out), _ptr(out_idx),
                                ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(x.device)), "fs_seg_map_reduce")
     return (out_map, out, out_idx) if op == "argmin" else (out_map, out)
+
+
+def scan_reduce(x, red: str = "add", scan: str = "add", out=None):
+    """NEXT-3, Fig 10c: reduce red (scan (+) x) in one read, the scan never materialised.
+    red in add (sum of prefix sums) / max / min (extreme prefix sum)."""
+    x = _dev(x, "x")
+    dt = _dt(x)
+    if out is None:
+        out = torch.empty((), dtype=x.dtype, device=x.device)
+    ws = workspace(_query(_lib.fs_scan_reduce_workspace, dt, x.numel()), x.device)
+    _ok(_lib.fs_scan_reduce(OPS[scan], OPS[red], dt, _ptr(x), x.numel(), _ptr(out), ctypes.c_void_p(ws.data_ptr()),
+                            ws.numel(), _stream(x.device)), "fs_scan_reduce")
+    return out
 
 
 def stream_red(vals, keys, k: int, sums=None, counts=None, with_counts: bool = True):

@@ -452,6 +452,29 @@ fs_status fs_seg_map_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t 
                               op.op == FS_ARGMIN ? out_idx : nullptr, ws, S(stream));
 }
 
+// ------------------------------------------------------------ NEXT-3: scan_reduce
+fs_status fs_scan_reduce_workspace(int32_t dtype, int64_t n, size_t *bytes) {
+    if (!bytes) return FS_ERR_NULL;
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (n < 0 || mul_overflows(n, 8)) return FS_ERR_SIZE;
+    *bytes = scan_reduce_ws(dtype);
+    return FS_OK;
+}
+
+fs_status fs_scan_reduce(int32_t scan_op, int32_t red_op, int32_t dtype, const void *in, int64_t n, void *out,
+                         void *ws, size_t ws_bytes, void *stream) {
+    size_t need = 0;
+    FS_TRY(fs_scan_reduce_workspace(dtype, n, &need));
+    if (scan_op != FS_ADD || (red_op != FS_ADD && red_op != FS_MAX && red_op != FS_MIN)) return FS_ERR_UNSUPPORTED;
+    if (!out || (n > 0 && !in)) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype);
+    if ((in && !aligned_to(in, es)) || !aligned_to(out, es)) return FS_ERR_UNSUPPORTED;
+    if (overlaps(out, es, in, n * es)) return FS_ERR_ALIAS;
+    FS_TRY(check_ws(ws, ws_bytes, need));
+    if (n > 0 && !aligned_to(in, 16)) return FS_ERR_UNSUPPORTED;  // 16-byte vector loads
+    return scan_reduce_run(red_op, dtype, in, n, out, ws, S(stream));
+}
+
 // ------------------------------------------------------------ utilities
 fs_status fs_check_device_error(void *ws, void *stream) {
     if (!ws) return FS_ERR_NULL;

@@ -93,6 +93,9 @@ fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, i
 size_t seg_map_reduce_ws(int op, int dt, int64_t nseg, int64_t L);
 fs_status seg_map_reduce_run(int op, int dt, const void *in, int64_t nseg, int64_t L, int64_t ci, float cf, void *ymap,
                              void *out, int64_t *out_idx, void *ws, cudaStream_t st);
+// scan_reduce.cu (NEXT-3)
+size_t scan_reduce_ws(int dt);
+fs_status scan_reduce_run(int red, int dt, const void *x, int64_t n, void *out, void *ws, cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 

@@ -180,6 +180,17 @@ def test_kmeans_step_validation(fs):
     assert fs.C.fs_kmeans_step_workspace(-1, 34, 32, ctypes.byref(sz)) == SIZE
 
 
+def test_scan_reduce_validation(fs):
+    big = 1 << 30
+    sr = fs.C.fs_scan_reduce
+    assert sr(1, 0, F32, P(FAKE_IN), 100, P(FAKE_OUT), P(FAKE_WS), big, None) == UNSUP   # scan op must be ADD
+    assert sr(0, 3, F32, P(FAKE_IN), 100, P(FAKE_OUT), P(FAKE_WS), big, None) == UNSUP   # no argmin reduce
+    assert sr(0, 0, F32, P(FAKE_IN), 100, P(FAKE_IN + 8), P(FAKE_WS), big, None) == ALIAS
+    assert sr(0, 0, F32, None, 100, P(FAKE_OUT), P(FAKE_WS), big, None) == NULL
+    assert sr(0, 0, F32, P(FAKE_IN), -1, P(FAKE_OUT), P(FAKE_WS), big, None) == SIZE
+    assert sr(0, 0, F32, P(FAKE_IN), 100, P(FAKE_OUT), None, 0, None) == WS
+
+
 def test_workspace_queries_and_regimes(fs):
     sz = ctypes.c_size_t(0)
     assert fs.C.fs_redomap_workspace(op(fs, 0, F32), 1 << 28, ctypes.byref(sz)) == OK and sz.value >= 256

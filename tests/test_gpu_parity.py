@@ -150,6 +150,37 @@ def test_kmeans_step_c3_kdd_and_ties(fs):
         _km_check(fs, small, cen, None, f"n={n}")
 
 
+# ------------------------------------------------------------------ NEXT-3: scan_reduce
+@pytest.mark.parametrize("n", [0, 1, 5, 127, 128, 4097, 1_000_003, 1 << 24])
+def test_scan_reduce(fs, n):
+    """Fig 10c fusion: reduce (scan x) in one pass, equal to the oracle's materialised scan +
+    reduce: integers bit-exact (wrap-around), f32 within 1e-4 of the f64 oracle relative to
+    the same computation on |x|."""
+    for dt in DTYPES:
+        for red in ("add", "max", "min"):
+            # add: full-range integers (wrap-around is exact); max/min: no prefix overflow
+            # (the max-prefix pair operator needs monotone addition, include/futseg.h)
+            full = np.dtype(dt).kind == "i" and red == "add"
+            x = workloads.full_range(n, n % 89, dt) if full else workloads.mixed(n, n % 89, dt)
+            got = host(fs.scan_reduce(cu(x), red))
+            want = oracle.scan_reduce(x, "add", red)
+            if dt == np.float32 and n == 0:
+                assert float(got) == float(want), (red, got, want)  # the neutral element
+            elif dt == np.float32:
+                scale = oracle.scan_reduce(np.abs(x), "add", "add") if red == "add" else np.abs(x).sum()
+                assert abs(float(got) - float(want)) <= 1e-4 * scale + 1e-30, (n, red, got, want)
+            else:
+                assert got == want, (n, dt, red, got, want)
+
+
+def test_scan_reduce_positive_closed_forms(fs):
+    """Closed forms on the GPU directly: prefix sums of ones; the max prefix of a +-1 walk."""
+    n = 1 << 20
+    assert int(host(fs.scan_reduce(torch.ones(n, dtype=torch.int64, device="cuda"), "add"))) == n * (n + 1) // 2
+    walk = np.where(np.arange(n) % 3 == 0, -1, 1).astype(np.int32)
+    assert int(host(fs.scan_reduce(cu(walk), "max"))) == int(np.cumsum(walk.astype(np.int64)).max())
+
+
 # ------------------------------------------------------------------ NEXT-4: seg_map_reduce
 @pytest.mark.parametrize("nseg,seglen", [(1, 1), (1000, 1), (777, 3), (4096, 4), (300, 32), (1000, 33), (64, 128),
                                          (50, 1000), (9, 4097), (3, 65537), (2, 1_000_003), (0, 5), (7, 0)])
