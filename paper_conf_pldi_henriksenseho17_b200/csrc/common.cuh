@@ -272,6 +272,7 @@ template <int N> __device__ __forceinline__ void bulk_wait() {
 // [0, 256)          : control words
 //     u32 ticket   @ 0     (single-counter kernels; reset by the last CTA)
 //     u32 err      @ 64    (device precondition flag, fs_check_device_error)
+//     u64 counters @ 128, 136, 192 (nn_knn barrier and candidates, kmeans delta)
 // [256, 16640)      : kWsMaxTickets u32 tickets (per column tile / per segment),
 //                     each reset to 0 by the CTA that consumes it
 // [16640, ...)      : per-primitive body (partials, scan tile states), never
@@ -280,6 +281,9 @@ template <int N> __device__ __forceinline__ void bulk_wait() {
 // zero-filled workspace stays valid across calls of different primitives.
 constexpr size_t kWsTicket = 0;
 constexpr size_t kWsErr = 64;
+constexpr size_t kWsCount0 = 128;  // u64 counters, zero between calls (reset by their last CTA):
+constexpr size_t kWsCount1 = 136;  //   nn_knn grid barrier / candidate count,
+constexpr size_t kWsCount2 = 192;  //   kmeans_step delta
 constexpr size_t kWsTickets = 256;
 constexpr int64_t kWsMaxTickets = 4096;
 constexpr size_t kWsHeader = kWsTickets + 4 * kWsMaxTickets;

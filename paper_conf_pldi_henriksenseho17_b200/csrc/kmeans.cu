@@ -420,7 +420,7 @@ static int64_t km_grid(int64_t n) {
 size_t kmeans_ws(int64_t n, int64_t d, int64_t k) {
     const int64_t G = (int64_t)sm_count() * 2;  // >= km_grid(n)
     (void)n;
-    return kWsHeader + 256 + align_up((size_t)G * k * d * 4, 256) + align_up((size_t)G * k * 4, 256);
+    return kWsHeader + align_up((size_t)G * k * d * 4, 256) + align_up((size_t)G * k * 4, 256);
 }
 
 template <int KS, int XR>
@@ -432,9 +432,9 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
     int64_t rows = n > 0 ? ceil_div(n, warps) : 0;
     rows = ceil_div(rows, kKmRS) * kKmRS;  // stages start 16-row (64d-byte) aligned
     char *w = (char *)ws;
-    unsigned long long *gdelta = (unsigned long long *)(w + kWsHeader);
-    float *parts = (float *)(w + kWsHeader + 256);
-    int *pcnt = (int *)(w + kWsHeader + 256 + align_up((size_t)G * k * d * 4, 256));
+    unsigned long long *gdelta = (unsigned long long *)(w + kWsCount2);  // zero between calls (header)
+    float *parts = (float *)(w + kWsHeader);
+    int *pcnt = (int *)(w + kWsHeader + align_up((size_t)G * k * d * 4, 256));
     const size_t smem = km_smem(d);
     cudaFuncSetAttribute((const void *)kmeans_step_kernel<KS, XR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)smem);

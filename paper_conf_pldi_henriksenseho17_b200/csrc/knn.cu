@@ -101,10 +101,10 @@ __device__ void knn_push(unsigned long long *S, KnnState *st, int kk, const unsi
 
 constexpr int kKnnBins = 4096;  // key >> 52: top 12 bits of the distance
 
-struct KnnCtl {          // in the workspace body (zero between calls)
-    unsigned barrier;    // grid barrier arrivals
-    unsigned ticket;     // CTAs done with phase B
-    unsigned long long ncand;
+struct KnnCtl {          // the workspace's self-resetting control words (zero between calls)
+    unsigned *barrier;   // grid barrier arrivals            (kWsCount0)
+    unsigned *ticket;    // CTAs done with phase B           (kWsTicket)
+    unsigned long long *ncand;  // candidates appended       (kWsCount1)
 };
 
 __device__ __forceinline__ unsigned long long knn_record_key(const float *lat, const float *lng, int64_t i, float q0,
@@ -114,7 +114,7 @@ __device__ __forceinline__ unsigned long long knn_record_key(const float *lat, c
 
 __global__ void __launch_bounds__(kKnnThreads, 1)
 knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t n, float q0, float q1, int kk,
-           int64_t chunk, KnnCtl *ctl, unsigned *ghist, unsigned long long *cand, float *out_dist,
+           int64_t chunk, KnnCtl ctl, unsigned *ghist, unsigned long long *cand, float *out_dist,
            int64_t *out_idx) {
     extern __shared__ __align__(16) unsigned long long S[];
     unsigned *hist = reinterpret_cast<unsigned *>(S);  // phase A/B alias of the sort buffer
@@ -144,8 +144,8 @@ knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t
     __syncthreads();
     if (tid == 0) {
         __threadfence();
-        atomicAdd(&ctl->barrier, 1u);
-        while (atomicAdd(&ctl->barrier, 0u) < gridDim.x) __nanosleep(64);
+        atomicAdd(ctl.barrier, 1u);
+        while (atomicAdd(ctl.barrier, 0u) < gridDim.x) __nanosleep(64);
         __threadfence();
     }
     __syncthreads();
@@ -191,7 +191,7 @@ knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t
             const unsigned mask = __ballot_sync(0xffffffffu, in);
             unsigned long long off = 0;
             if (mask) {
-                if (lane == 0) off = atomicAdd(&ctl->ncand, (unsigned long long)__popc(mask));
+                if (lane == 0) off = atomicAdd(ctl.ncand, (unsigned long long)__popc(mask));
                 off = __shfl_sync(0xffffffffu, off, 0);
             }
             if (in) __stcg(cand + off + __popc(mask & ((1u << lane) - 1u)), key);
@@ -200,7 +200,7 @@ knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t
     __syncthreads();
     if (tid == 0) {
         __threadfence();
-        last = atomicAdd(&ctl->ticket, 1u) == gridDim.x - 1;
+        last = atomicAdd(ctl.ticket, 1u) == gridDim.x - 1;
         if (last) __threadfence();
     }
     __syncthreads();
@@ -212,7 +212,7 @@ knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t
         st.T = kKeyInf;
     }
     __syncthreads();
-    const int64_t total = (int64_t)__ldcg(&ctl->ncand);
+    const int64_t total = (int64_t)__ldcg(ctl.ncand);
     for (int64_t b = 0; b < total; b += kKnnTile) {
         unsigned long long key[kKnnPer];
         bool valid[kKnnPer];
@@ -236,16 +236,14 @@ knn_kernel(const float *__restrict__ lat, const float *__restrict__ lng, int64_t
     }
     for (int b = tid; b < kKnnBins; b += kKnnThreads) ghist[b] = 0;  // leave the workspace reusable
     if (tid == 0) {
-        ctl->barrier = 0;
-        ctl->ticket = 0;
-        ctl->ncand = 0;
+        *ctl.barrier = 0;
+        *ctl.ticket = 0;
+        *ctl.ncand = 0;
     }
 }
 
-// workspace body: [KnnCtl | pad to 256] [histogram 4096 u32] [candidates: n u64]
-size_t knn_ws(int64_t n) {
-    return kWsHeader + 256 + (size_t)kKnnBins * 4 + align_up((size_t)(n > 0 ? n : 1) * 8, 256);
-}
+// workspace body: [candidates: n u64]
+size_t knn_ws(int64_t n) { return kWsHeader + align_up((size_t)(n > 0 ? n : 1) * 8, 256); }
 
 fs_status knn_run(const float *lat, const float *lng, int64_t n, float q0, float q1, int64_t kk, float *out_dist,
                   int64_t *out_idx, void *ws, cudaStream_t st) {
@@ -261,9 +259,13 @@ fs_status knn_run(const float *lat, const float *lng, int64_t n, float q0, float
     if (G < 1) G = 1;
     int64_t chunk = n > 0 ? ceil_div(n, G) : 0;
     char *w = (char *)ws;
-    KnnCtl *ctl = (KnnCtl *)(w + kWsHeader);
-    unsigned *ghist = (unsigned *)(w + kWsHeader + 256);
-    unsigned long long *cand = (unsigned long long *)(w + kWsHeader + 256 + (size_t)kKnnBins * 4);
+    // counters and histogram live in the workspace's zero-between-calls header (control
+    // words; the 4096 self-resetting ticket slots hold the histogram), reset by the last CTA;
+    // the body (candidates) is never assumed zero
+    static_assert(kKnnBins == kWsMaxTickets, "histogram = the ticket slots");
+    KnnCtl ctl{(unsigned *)(w + kWsCount0), (unsigned *)(w + kWsTicket), (unsigned long long *)(w + kWsCount1)};
+    unsigned *ghist = (unsigned *)(w + kWsTickets);
+    unsigned long long *cand = (unsigned long long *)(w + kWsHeader);
     int kki = (int)kk;
     void *args[] = {(void *)&lat, (void *)&lng, (void *)&n, (void *)&q0, (void *)&q1, (void *)&kki, (void *)&chunk,
                     (void *)&ctl, (void *)&ghist, (void *)&cand, (void *)&out_dist, (void *)&out_idx};

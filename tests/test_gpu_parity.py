@@ -150,6 +150,46 @@ def test_kmeans_step_c3_kdd_and_ties(fs):
         _km_check(fs, small, cen, None, f"n={n}")
 
 
+# ------------------------------------------------------------------ workspace contract
+def test_dirty_workspace_body(fs):
+    """The workspace body (past the control words and self-resetting tickets) is never
+    assumed zero: fill it with garbage before every primitive and compare with the oracle."""
+    HDR = 256 + 4 * 4096
+
+    def dirty():
+        ws = fs.workspace(1 << 26, "cuda")
+        ws[HDR:].fill_(0xA5)
+        torch.cuda.synchronize()
+
+    lat, lng, q = workloads.c2_nn(base=20_000, reps=3)
+    dirty()
+    d, i = fs.nn_knn(cu(lat), cu(lng), q, 100)
+    np.testing.assert_array_equal(host(i), oracle.nn_knn(lat, lng, q, 100)[1])
+    pts, _ = workloads.c3_kmeans(n=40_000, d=34, k=32)
+    prev = workloads.ints(40_000, 3, 0, 32)
+    dirty()
+    m, _, cnt, _, dl = fs.kmeans_step(cu(pts), cu(pts[:32].copy()), prev=cu(prev))
+    wm, _, wc, _, wd = oracle.kmeans_step(pts, pts[:32].copy(), prev)
+    np.testing.assert_array_equal(host(m), wm)
+    np.testing.assert_array_equal(host(cnt), wc)
+    assert int(host(dl)[0]) == wd
+    x = workloads.mixed(3 * 70_001, 5, np.int32)
+    dirty()
+    mp, rs = fs.seg_map_reduce(cu(x), 3, 70_001, 2, "add")
+    np.testing.assert_array_equal(host(rs), oracle.seg_map_reduce(x, 3, 70_001, 2, "add")[1])
+    dirty()
+    assert int(host(fs.scan_reduce(cu(x), "add"))) == int(oracle.scan_reduce(x, "add", "add"))
+    dirty()
+    assert int(host(fs.redomap(cu(x), "add"))) == int(oracle.reduce(x, "add"))
+    dirty()
+    np.testing.assert_array_equal(host(fs.scanomap(cu(x), "add")), oracle.scan(x, "add"))
+    dirty()
+    np.testing.assert_array_equal(host(fs.seg_reduce(cu(x), 3, 70_001, "max")), oracle.seg_reduce(x, 3, 70_001, "max"))
+    dirty()
+    s_, c_ = fs.stream_red(cu(pts), cu(prev), 32)
+    np.testing.assert_array_equal(host(c_), oracle.stream_red(pts, prev, 32)[1])
+
+
 # ------------------------------------------------------------------ NEXT-3: scan_reduce
 @pytest.mark.parametrize("n", [0, 1, 5, 127, 128, 4097, 1_000_003, 1 << 24])
 def test_scan_reduce(fs, n):
