@@ -196,6 +196,13 @@ fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen
 fs_status fs_transpose_2d(int32_t dtype, const void *in, int64_t rows, int64_t cols, void *out,
                           void *stream);
 
+/* new_centres[c][j] = counts[c] > 0 ? sums[c][j] / counts[c] : centres[c][j] (R19): the
+ * last step of fs_kmeans_step, on its own for sums and counts that were first combined
+ * across GPUs (one all_reduce, multi-GPU layer).  k*d f32 / k int32, device pointers;
+ * new_centres must not overlap the inputs.  No workspace. */
+fs_status fs_kmeans_finish(const float *sums, const int32_t *counts, const float *centres, int64_t k, int64_t d,
+                           float *new_centres, void *stream);
+
 /* ---------------------------------------------------------------- NEXT-2: nn_knn */
 /* Rodinia NN's kk nearest neighbours: "100 reduce operations for finding the
  * nearest neighbors", the reduce computing "both the minimal value and the

@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "kmeans_step", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -77,6 +77,7 @@ _SIG = {
     "fs_seg_map_reduce": [fs_opdesc, _P, _L, _L, _L, ctypes.c_float, _P, _P, _P, _P, ctypes.c_size_t, _P],
     "fs_scan_reduce_workspace": [_I, _L, _SZ],
     "fs_scan_reduce": [_I, _I, _I, _P, _L, _P, _P, ctypes.c_size_t, _P],
+    "fs_kmeans_finish": [_P, _P, _P, _L, _L, _P, _P],
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
@@ -310,6 +311,16 @@ def seg_map_reduce(x, nseg: int, seglen: int, c, op: str = "add", out_map=None, 
     _ok(_lib.fs_seg_map_reduce(o, _ptr(x), nseg, seglen, ci, float(c), _ptr(out_map), _ptr(out), _ptr(out_idx),
                                ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(x.device)), "fs_seg_map_reduce")
     return (out_map, out, out_idx) if op == "argmin" else (out_map, out)
+
+
+def kmeans_finish(sums, counts, centres, out=None):
+    """new centres = sums / counts, an empty cluster keeps its centre (R19)."""
+    sums, counts, centres = _dev(sums, "sums"), _dev(counts, "counts"), _dev(centres, "centres")
+    k, d = centres.shape
+    out = torch.empty_like(centres) if out is None else out
+    _ok(_lib.fs_kmeans_finish(_ptr(sums), _ptr(counts), _ptr(centres), k, d, _ptr(out), _stream(sums.device)),
+        "fs_kmeans_finish")
+    return out
 
 
 def scan_reduce(x, red: str = "add", scan: str = "add", out=None):

@@ -452,6 +452,20 @@ fs_status fs_seg_map_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t 
                               op.op == FS_ARGMIN ? out_idx : nullptr, ws, S(stream));
 }
 
+fs_status fs_kmeans_finish(const float *sums, const int32_t *counts, const float *centres, int64_t k, int64_t d,
+                           float *new_centres, void *stream) {
+    if (k < 0 || d < 0 || mul_overflows(k, d)) return FS_ERR_SIZE;
+    if (k * d == 0) return FS_OK;
+    if (!sums || !counts || !centres || !new_centres) return FS_ERR_NULL;
+    if (!aligned_to(sums, 4) || !aligned_to(counts, 4) || !aligned_to(centres, 4) || !aligned_to(new_centres, 4))
+        return FS_ERR_UNSUPPORTED;
+    const int64_t b = k * d * 4;
+    if (overlaps(new_centres, b, sums, b) || overlaps(new_centres, b, centres, b) ||
+        overlaps(new_centres, b, counts, k * 4))
+        return FS_ERR_ALIAS;
+    return kmeans_finish_run(sums, counts, centres, k, d, new_centres, S(stream));
+}
+
 // ------------------------------------------------------------ NEXT-3: scan_reduce
 fs_status fs_scan_reduce_workspace(int32_t dtype, int64_t n, size_t *bytes) {
     if (!bytes) return FS_ERR_NULL;

@@ -96,6 +96,8 @@ fs_status seg_map_reduce_run(int op, int dt, const void *in, int64_t nseg, int64
 // scan_reduce.cu (NEXT-3)
 size_t scan_reduce_ws(int dt);
 fs_status scan_reduce_run(int red, int dt, const void *x, int64_t n, void *out, void *ws, cudaStream_t st);
+fs_status kmeans_finish_run(const float *sums, const int32_t *counts, const float *cen, int64_t k, int64_t d,
+                            float *new_cen, cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 

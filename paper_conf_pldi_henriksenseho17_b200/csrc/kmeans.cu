@@ -459,4 +459,21 @@ fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, i
     return FS_ERR_UNSUPPORTED;
 }
 
+// new centres from (already combined) sums and counts: the last step of the iteration
+// when the sums are reduced across GPUs first (dist.kmeans_step); R19 for empty clusters
+__global__ void kmeans_finish_kernel(const float *sums, const int32_t *counts, const float *cen, int64_t k, int64_t d,
+                                     float *new_cen) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < k * d; e += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t c = counts[e / d];
+        new_cen[e] = c > 0 ? __fdiv_rn(sums[e], (float)c) : cen[e];
+    }
+}
+
+fs_status kmeans_finish_run(const float *sums, const int32_t *counts, const float *cen, int64_t k, int64_t d,
+                            float *new_cen, cudaStream_t st) {
+    const int64_t kd = k * d;
+    kmeans_finish_kernel<<<(unsigned)(kd > 0 ? ceil_div(kd, 256) : 1), 256, 0, st>>>(sums, counts, cen, k, d, new_cen);
+    return launch_status();
+}
+
 }  // namespace fs

@@ -11,7 +11,9 @@ one NCCL allreduce over NVLink").
               carry = combine of the totals of ranks < r (F5's accumulator a,
               L1071-1074) -> local scanomap with carry-in
   stream_red  rows sharded; local chunk results combined by all_reduce (map(+))
-  seg_reduce, seg_scan, transpose_2d
+  kmeans_step (NEXT-1) points sharded; fused local step, one all_reduce of
+              (sums, counts, delta), new centres from the global sums
+  seg_reduce, seg_scan, transpose_2d, seg_map_reduce (NEXT-4)
               outer segments / row blocks sharded; no collective
 
 The collectives go through ``torch.distributed`` (NCCL over NVLink on GPUs,
@@ -93,6 +95,25 @@ def stream_red(vals_local, keys_local, k: int, group=None, backend=None):
     dist.all_reduce(sums, op=dist.ReduceOp.SUM, group=group)
     dist.all_reduce(counts, op=dist.ReduceOp.SUM, group=group)
     return sums, counts
+
+
+def kmeans_step(points_local, centres, prev_local=None, group=None, backend=None):
+    """One K-means iteration over every rank's points (NEXT-1): the fused local step on the
+    shard, then ONE exchange -- all_reduce of the partial sums, counts and changed-label
+    count -- and the new centres from the global sums (fs_kmeans_finish).  Returns
+    (membership of the local points, sums, counts, new centres, delta)."""
+    be = backend or _default_backend()
+    m, sums, counts, _, delta = be.kmeans_step(points_local, centres, prev=prev_local)
+    dist.all_reduce(sums, op=dist.ReduceOp.SUM, group=group)
+    dist.all_reduce(counts, op=dist.ReduceOp.SUM, group=group)
+    dist.all_reduce(delta, op=dist.ReduceOp.SUM, group=group)
+    return m, sums, counts, be.kmeans_finish(sums, counts, centres), delta
+
+
+def seg_map_reduce(x_local, nseg_local: int, seglen: int, c, op="add", backend=None):
+    """NEXT-4 rows sharded (rank r owns a block of rows): no exchange."""
+    be = backend or _default_backend()
+    return be.seg_map_reduce(x_local, nseg_local, seglen, c, op)
 
 
 def seg_reduce(x_local, nseg_local: int, seglen: int, op="add", layout="row", backend=None):

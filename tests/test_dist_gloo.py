@@ -69,6 +69,19 @@ class OracleShim:
     def transpose_2d(self, x):
         return torch.from_numpy(oracle.transpose_2d(x.numpy()))
 
+    def kmeans_step(self, pts, cen, prev=None):
+        m, s, c, n, d = oracle.kmeans_step(pts.numpy(), cen.numpy(), None if prev is None else prev.numpy())
+        return (torch.from_numpy(m), torch.from_numpy(s.astype(np.float32)), torch.from_numpy(c),
+                torch.from_numpy(n.astype(np.float32)), torch.tensor([d], dtype=torch.int64))
+
+    def kmeans_finish(self, sums, counts, cen):
+        c = counts.numpy()[:, None]
+        return torch.from_numpy(np.where(c > 0, sums.numpy() / np.maximum(c, 1), cen.numpy()).astype(np.float32))
+
+    def seg_map_reduce(self, x, nseg, seglen, c, op="add"):
+        r = oracle.seg_map_reduce(x.numpy(), nseg, seglen, c, op)
+        return tuple(torch.from_numpy(np.asarray(v)) for v in r)
+
 
 def _free_port():
     s = socket.socket()
@@ -121,6 +134,24 @@ def _worker(rank, world, port, fails):
         ws, wc = oracle.stream_red(pts, mem, 5)
         np.testing.assert_array_equal(counts.numpy(), wc)
         np.testing.assert_allclose(sums.numpy(), ws, rtol=1e-5)
+        # ---- one K-means iteration over sharded points: local fused step + one all_reduce
+        prev = workloads.ints(pts.shape[0], 8, 0, 5)
+        cen = pts[:5].copy()
+        m, ks, kc, kn, kd = fd.kmeans_step(torch.from_numpy(pts[lo:hi].copy()), torch.from_numpy(cen),
+                                           prev_local=torch.from_numpy(prev[lo:hi].copy()), backend=be)
+        wm, wsum, wcnt, wnew, wdel = oracle.kmeans_step(pts, cen, prev)
+        np.testing.assert_array_equal(m.numpy(), wm[lo:hi])
+        np.testing.assert_array_equal(kc.numpy(), wcnt)
+        assert int(kd.item()) == wdel
+        np.testing.assert_allclose(ks.numpy(), wsum, rtol=1e-5)
+        np.testing.assert_allclose(kn.numpy(), wnew, rtol=1e-5)
+        # ---- NEXT-4 row nest, rows sharded
+        xr = workloads.mixed(50 * 33, 6, np.float32)
+        rlo2, rhi2 = fd.shard_range(50, rank, world)
+        mp, rs = fd.seg_map_reduce(torch.from_numpy(xr[rlo2 * 33:rhi2 * 33].copy()), rhi2 - rlo2, 33, 1.0, backend=be)
+        wmp, wrs = oracle.seg_map_reduce(xr, 50, 33, 1.0)
+        np.testing.assert_array_equal(mp.numpy(), wmp[rlo2 * 33:rhi2 * 33])
+        np.testing.assert_allclose(rs.numpy(), wrs[rlo2:rhi2], rtol=1e-6)
         # ---- outer segments sharded, no exchange
         nseg, L = 101, 37
         xs = workloads.mixed(nseg * L, 4, np.int32)

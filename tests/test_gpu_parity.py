@@ -253,6 +253,17 @@ def test_seg_map_reduce_misaligned(fs):
     assert_reduced(got[1], want[1], "add", oracle.seg_reduce(np.abs(x), 37, 1001, "add"), "misaligned")
 
 
+def test_kmeans_finish_matches_fused(fs):
+    """fs_kmeans_finish (the multi-GPU layer's last step) = the fused step's own division,
+    bit for bit; an empty cluster keeps its centre."""
+    pts, _ = workloads.c3_kmeans(n=60_000, d=34, k=8)
+    cen = np.concatenate([pts[:7], np.full((1, 34), 9.0, np.float32)])
+    m, sums, counts, newc, _ = fs.kmeans_step(cu(pts), cu(cen))
+    fin = fs.kmeans_finish(sums, counts, cu(cen))
+    np.testing.assert_array_equal(host(fin), host(newc))
+    assert int(host(counts)[7]) == 0 and np.all(host(fin)[7] == 9.0)
+
+
 # ------------------------------------------------------------------ NEXT-2: nn_knn
 def _knn_check(fs, lat, lng, q, kk, off=0):
     d, i = fs.nn_knn(cu(lat, off), cu(lng, off), q, kk)
