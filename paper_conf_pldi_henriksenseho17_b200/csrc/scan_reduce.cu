@@ -10,7 +10,8 @@
 // Both products are associative (not commutative), so chunks may run in parallel as
 // long as they are combined in index order -- the q = 1 stream_seq of Fig 10c in every
 // lane (registers only), then ordered shuffle trees, then warps in order.
-//   lane : its 16-byte vector of a 32-vector tile, folded sequentially;
+//   lane : its 8 contiguous elements (two or four 16-byte vectors) of a tile, folded
+//          sequentially;
 //   warp : ordered tree over the 32 lanes, then the tile joins the warp's running pair;
 //          a warp owns one contiguous chunk of tiles;
 //   last CTA (ticket): the warps' pairs in order (f64 for f32) -> the result.
@@ -87,19 +88,23 @@ scan_reduce_kernel(const T *__restrict__ x, int64_t n, int64_t tiles_per_warp, S
     using C = std::conditional_t<std::is_floating_point<T>::value, double, T>;
     using FC = SRFuse<RED, C>;
     constexpr int VEC = 16 / sizeof(T);
-    constexpr int64_t TILE = 32 * VEC;
+    constexpr int PV = 8 / VEC;             // 16-byte vectors per lane: 8 contiguous elements
+    constexpr int E = PV * VEC;
+    constexpr int64_t TILE = 32 * E;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t gw = (int64_t)blockIdx.x * 8 + warp;
     const int64_t ntiles = (n + TILE - 1) / TILE;
     const int64_t t0 = gw * tiles_per_warp, t1 = min(ntiles, t0 + tiles_per_warp);
     SRPair<T> run = F::id();
-    int4 r[U], rn[U];
-    auto load = [&](int64_t tb, int4 (&dst)[U]) {
+    int4 r[U][PV], rn[U][PV];
+    auto load = [&](int64_t tb, int4 (&dst)[U][PV]) {
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int64_t e0 = (tb + u) * TILE + (int64_t)lane * VEC;
-            if (tb + u < t1 && e0 + VEC <= n) dst[u] = ldg16(x + e0);
-        }
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int v = 0; v < PV; ++v) {
+                const int64_t e0 = (tb + u) * TILE + (int64_t)lane * E + v * VEC;
+                if (tb + u < t1 && e0 + VEC <= n) dst[u][v] = ldg16(x + e0);
+            }
     };
     if (t0 < t1) load(t0, r);
     for (int64_t t = t0; t < t1; t += U) {
@@ -107,22 +112,30 @@ scan_reduce_kernel(const T *__restrict__ x, int64_t n, int64_t tiles_per_warp, S
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             if (t + u >= t1) break;  // warp-uniform
-            const int64_t e0 = (t + u) * TILE + (int64_t)lane * VEC;
-            if (e0 + VEC <= n && (t + u + 1) * TILE <= n) {
-                // full tile: every lane holds VEC elements, so every block length in the
-                // ordered tree is static -- the pair is (A, R) and L is implicit
-                const Vec16<T> e = as_vec<T>(r[u]);
-                T a = e.e[0], rr = e.e[0];
+            const int64_t e0 = (t + u) * TILE + (int64_t)lane * E;
+            if ((t + u + 1) * TILE <= n) {
+                // full tile: every lane holds E contiguous elements, so every block length in
+                // the ordered tree is static -- the pair is (A, R) and L is implicit
+                T a, rr;
 #pragma unroll
-                for (int k = 1; k < VEC; ++k) {
-                    a = wrap_add(a, e.e[k]);
-                    rr = RED == kAdd ? wrap_add(rr, a) : (RED == kMax ? (rr < a ? a : rr) : (a < rr ? a : rr));
+                for (int v = 0; v < PV; ++v) {
+                    const Vec16<T> ev = as_vec<T>(r[u][v]);
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) {
+                        if (v == 0 && k == 0) {
+                            a = rr = ev.e[0];
+                        } else {
+                            a = wrap_add(a, ev.e[k]);
+                            rr = RED == kAdd ? wrap_add(rr, a)
+                                             : (RED == kMax ? (rr < a ? a : rr) : (a < rr ? a : rr));
+                        }
+                    }
                 }
 #pragma unroll
                 for (int off = 1; off < 32; off <<= 1) {
                     const T a2 = shfl_down_v(a, off), r2 = shfl_down_v(rr, off);
                     if ((lane & (2 * off - 1)) == 0) {
-                        if (RED == kAdd) rr = wrap_add(wrap_add(rr, r2), F::mulw((int64_t)VEC * off, a));
+                        if (RED == kAdd) rr = wrap_add(wrap_add(rr, r2), F::mulw((int64_t)E * off, a));
                         else {
                             const T c = wrap_add(a, r2);
                             rr = RED == kMax ? (rr < c ? c : rr) : (c < rr ? c : rr);
@@ -133,15 +146,10 @@ scan_reduce_kernel(const T *__restrict__ x, int64_t n, int64_t tiles_per_warp, S
                 run = F::comb(run, SRPair<T>{__shfl_sync(0xffffffffu, a, 0), __shfl_sync(0xffffffffu, rr, 0), TILE});
                 continue;
             }
-            Vec16<T> e;
-            int cnt = VEC;
-            if (e0 + VEC <= n) {
-                e = as_vec<T>(r[u]);
-            } else {  // ragged end of the array
-                cnt = e0 < n ? (int)(n - e0) : 0;
-                for (int k = 0; k < VEC; ++k) e.e[k] = k < cnt ? x[e0 + k] : T(0);
-            }
-            SRPair<T> p = sr_lift_vec<RED, T>(e, cnt);
+            // ragged end of the array: element by element
+            SRPair<T> p = F::id();
+            for (int k = 0; k < E; ++k)
+                if (e0 + k < n) p = F::comb(p, SRPair<T>{x[e0 + k], x[e0 + k], 1});
             // ordered tree: lane i absorbs lane i + off (its right neighbour block)
 #pragma unroll
             for (int off = 1; off < 32; off <<= 1) {
@@ -152,7 +160,9 @@ scan_reduce_kernel(const T *__restrict__ x, int64_t n, int64_t tiles_per_warp, S
                                          __shfl_sync(0xffffffffu, p.L, 0)});
         }
 #pragma unroll
-        for (int u = 0; u < U; ++u) r[u] = rn[u];
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int v = 0; v < PV; ++v) r[u][v] = rn[u][v];
     }
     __shared__ bool last;
     if (lane == 0) wparts[gw] = run;
@@ -197,10 +207,10 @@ size_t scan_reduce_ws(int dt) {
 
 template <int RED, typename T>
 static fs_status sr_launch(const void *x, int64_t n, void *out, void *ws, cudaStream_t st) {
-    constexpr int64_t TILE = 32 * (16 / sizeof(T));
+    constexpr int64_t TILE = 32 * 8;  // 8 contiguous elements per lane
     const int64_t ntiles = ceil_div(n > 0 ? n : 1, TILE);
     // exactly the resident CTAs (one wave: every warp's chunk runs concurrently), <= 8 per SM
-    int64_t G = resident_blocks((const void *)scan_reduce_kernel<RED, T, 4>, 256);
+    int64_t G = resident_blocks((const void *)scan_reduce_kernel<RED, T, 2>, 256);
     if (G > (int64_t)sm_count() * 8) G = (int64_t)sm_count() * 8;
     int64_t tpw = ceil_div(ntiles, G * 8);
     if (tpw < 4) {  // small inputs: fewer warps, >= 4 tiles each
@@ -208,7 +218,7 @@ static fs_status sr_launch(const void *x, int64_t n, void *out, void *ws, cudaSt
         G = ceil_div(ceil_div(ntiles, tpw), 8);
     }
     char *w = (char *)ws;
-    scan_reduce_kernel<RED, T, 4><<<(unsigned)G, 256, 0, st>>>((const T *)x, n, tpw, (SRPair<T> *)(w + kWsHeader),
+    scan_reduce_kernel<RED, T, 2><<<(unsigned)G, 256, 0, st>>>((const T *)x, n, tpw, (SRPair<T> *)(w + kWsHeader),
                                                               (unsigned *)(w + kWsTicket), (T *)out);
     return launch_status();
 }
