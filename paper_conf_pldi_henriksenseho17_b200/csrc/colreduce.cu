@@ -88,12 +88,15 @@ colreduce_kernel(const T *__restrict__ x, int64_t m, int64_t w, int CG, int64_t 
         }
     }
     if (single) return;
-    __threadfence();
+    // the barrier orders the CTA's partial stores before thread 0's cumulative gpu fence
     __syncthreads();
-    if (t == 0) last = atomicAdd(tickets + blockIdx.x, 1u) == gridDim.y - 1;
+    if (t == 0) {
+        __threadfence();
+        last = atomicAdd(tickets + blockIdx.x, 1u) == gridDim.y - 1;
+        if (last) __threadfence();
+    }
     __syncthreads();
     if (!last) return;
-    __threadfence();
     // last CTA of this column tile: fold the gridDim.y partial rows (fixed order)
     const int Y = gridDim.y;
     const int tcw = (int)((w - col0) < TCW ? (w - col0) : TCW);

@@ -30,10 +30,10 @@ __device__ __forceinline__ void finish_grid(typename O::V acc, typename O::V *pa
         __threadfence();
         unsigned t = atomicAdd(ticket, 1u);
         last = (t == gridDim.x - 1);
+        if (last) __threadfence();  // acquire: one fence, ordered for the CTA by the barrier
     }
     __syncthreads();
     if (!last) return;
-    __threadfence();
     V a = O::id();
     for (int i = threadIdx.x; i < (int)gridDim.x; i += NT) a = O::comb(a, ld_cg(partials + i));
     a = block_reduce<O, NT>(a, sm);

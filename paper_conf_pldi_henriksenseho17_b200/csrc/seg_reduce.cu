@@ -332,10 +332,10 @@ seg_block_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, int64_t C, in
             st_cg(partials + it, a);
             __threadfence();
             last = atomicAdd(tickets + s, 1u) == (unsigned)(C - 1);
+            if (last) __threadfence();  // acquire, ordered for the CTA by the barrier
         }
         __syncthreads();
         if (last) {
-            __threadfence();
             V b = O::id();
             for (int64_t q = t; q < C; q += NT) b = O::comb(b, ld_cg(partials + s * C + q));
             b = block_reduce<O, NT>(b, sm);
