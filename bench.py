@@ -188,13 +188,15 @@ def make_step(fs, W, world):
 
 # ------------------------------------------------------------------ SURVEY 8(f) "next" rows
 def time_next_rows(fs, W, dev, K, peak):
-    """Each NEXT row timed on its own (CUDA events, K reps, L2 flushed before every rep by
-    a 1 GB write outside the events).  Not part of the step value (8(a) rows only)."""
+    """Each NEXT row timed on its own (one warm-up call, then CUDA events over K reps, L2
+    flushed before every rep by a 1 GB write outside the events; median and min reported).
+    Not part of the step value (8(a) rows only)."""
     import torch
     flush = torch.empty(1 << 30, dtype=torch.uint8, device=dev)  # ~150 us of GPU time: the host stays ahead
     rows = {}
 
     def timed(fn, reps=K):
+        fn()  # warm-up: workspace growth, function attributes
         ms = []
         for _ in range(reps):
             flush.zero_()
@@ -204,7 +206,7 @@ def time_next_rows(fs, W, dev, K, peak):
             b.record()
             b.synchronize()
             ms.append(a.elapsed_time(b))
-        return sum(ms) / len(ms), min(ms)
+        return statistics.median(ms), min(ms)
 
     # NEXT-2: NN's 100 argmin rounds (L1653-1655) as one selection launch
     nn, kk = W["lat"].numel(), 100

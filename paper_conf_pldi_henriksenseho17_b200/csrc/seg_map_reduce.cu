@@ -8,6 +8,7 @@
 // reduction separately).  Per 16-byte vector: load once, store x + c, fold x.
 //   short rows (L = 2^j <= 32 vectors, aligned): grid-stride over vectors; a row is G
 //     consecutive lanes (or part of one vector), reduced with xor shuffles (as KG0);
+//   long rows (L >= 8192) and enough of them: a CTA per row (a compact read window);
 //   otherwise: a warp per (row, piece); a row longer than the machine's warps can cover
 //     one per row is cut into C pieces whose partials the last piece (per-row ticket)
 //     combines in piece order (deterministic), as KG4.
@@ -164,8 +165,68 @@ segmr_warp_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, int64_t C, i
     }
 }
 
+// a CTA per long row (L >= 8192, rows enough to fill the machine): all 256 threads stream
+// the same row, so the GPU reads a compact window of the matrix at any moment
+template <int OP, typename T, int U>
+__global__ void __launch_bounds__(256)
+segmr_block_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T c, bool vstore, T *__restrict__ ymap,
+                   T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    __shared__ V sm[32];
+    const int t = threadIdx.x;
+    for (int64_t s = blockIdx.x; s < nseg; s += gridDim.x) {
+        const T *p = x + s * L;
+        T *q = ymap + s * L;
+        int64_t head = (int64_t)(((16 - ((uintptr_t)p & 15)) & 15) / sizeof(T));
+        if (head > L) head = L;
+        const int64_t nvec = (L - head) / VEC, tail0 = head + nvec * VEC;
+        V a = O::id();
+        if (t < head) {
+            const T xv = __ldg(p + t);
+            q[t] = map_add(xv, c);
+            a = O::fold(a, xv, t);
+        }
+        const int4 *pv = reinterpret_cast<const int4 *>(p + head);
+        for (int64_t v = t; v < nvec; v += (int64_t)U * 256) {
+            int4 r[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (v + u * 256 < nvec) r[u] = ldg16(pv + v + u * 256);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t vv = v + u * 256;
+                if (vv >= nvec) break;
+                const Vec16<T> e = as_vec<T>(r[u]);
+                Vec16<T> o;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) o.e[k] = map_add(e.e[k], c);
+                T *qo = q + head + vv * VEC;
+                if (vstore) {
+                    *reinterpret_cast<int4 *>(qo) = *reinterpret_cast<const int4 *>(&o);
+                } else {
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) qo[k] = o.e[k];
+                }
+                const int64_t b = head + vv * VEC;
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], b + k);
+            }
+        }
+        if (t < L - tail0) {
+            const T xv = __ldg(p + tail0 + t);
+            q[tail0 + t] = map_add(xv, c);
+            a = O::fold(a, xv, tail0 + t);
+        }
+        a = block_reduce<O, 256>(a, sm);
+        if (t == 0) store_out<O>(out, out_idx, s, a);
+        __syncthreads();  // sm reuse
+    }
+}
+
 struct SegMrPlan {
-    bool shortp;
+    bool shortp, block;
     int64_t C, CS, grid;
 };
 
@@ -174,8 +235,9 @@ static SegMrPlan segmr_plan(int dt, int64_t nseg, int64_t L, bool aligned) {
     const int64_t vec = 16 / (int64_t)dtype_size(dt);
     p.shortp = aligned && nseg > 0 && L >= 1 && L <= 32 * vec && (L & (L - 1)) == 0;
     const int64_t warps = (int64_t)sm_count() * 64;
+    p.block = !p.shortp && L >= 8192 && nseg >= 4 * (int64_t)sm_count();
     p.C = 1;
-    if (!p.shortp && nseg > 0 && nseg < 8 * warps && L > 2048) {  // >= ~8 items per warp: no tail
+    if (!p.shortp && !p.block && nseg > 0 && nseg < 8 * warps && L > 2048) {  // >= ~8 items per warp: no tail
         p.C = ceil_div(8 * warps, nseg);
         const int64_t maxc = ceil_div(L, 2048);  // pieces of >= 2048 elements
         if (p.C > maxc) p.C = maxc;
@@ -214,6 +276,13 @@ template <int OP, typename T> struct SegMrRun {
             return launch_status();
         }
         const bool vstore = ((((uintptr_t)in) ^ ((uintptr_t)ymap)) & 15) == 0;
+        if (p.block) {
+            auto kb = segmr_block_kernel<OP, T, 4>;
+            int64_t grid = resident_blocks((const void *)kb, 256);
+            grid = grid > nseg ? nseg : grid;
+            kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in, nseg, L, c, vstore, (T *)ymap, (T *)out, out_idx);
+            return launch_status();
+        }
         char *w = (char *)ws;
         V *parts = (V *)(w + kWsHeader);
         unsigned *tickets = (unsigned *)(w + kWsHeader + align_up((size_t)nseg * p.C * sizeof(V), 256));

@@ -223,7 +223,8 @@ def test_scan_reduce_positive_closed_forms(fs):
 
 # ------------------------------------------------------------------ NEXT-4: seg_map_reduce
 @pytest.mark.parametrize("nseg,seglen", [(1, 1), (1000, 1), (777, 3), (4096, 4), (300, 32), (1000, 33), (64, 128),
-                                         (50, 1000), (9, 4097), (3, 65537), (2, 1_000_003), (0, 5), (7, 0)])
+                                         (50, 1000), (9, 4097), (3, 65537), (2, 1_000_003), (0, 5), (7, 0),
+                                         (700, 8192), (601, 10_001)])
 def test_seg_map_reduce(fs, nseg, seglen):
     """L247-252 fused row nest: x + c written and each row reduced in one read; every op,
     all dtypes, short power-of-two rows (shuffle groups), warp rows, rows cut into pieces."""
