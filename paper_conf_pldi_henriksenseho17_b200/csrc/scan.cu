@@ -131,20 +131,6 @@ template <class S> struct TileState<S, false> {
 constexpr int kScanThreads = FS_SCAN_NT;
 constexpr unsigned kStAgg = 1, kStIncl = 2;
 
-// -DFS_SCAN_PROFILE: thread 0 of every CTA accumulates clock64 cycles per phase of
-// scan_pipe_kernel into fs_scan_prof[] (debug / ncu-free attribution only)
-#ifdef FS_SCAN_PROFILE
-__device__ unsigned long long fs_scan_prof[16];
-}  // namespace fs
-extern "C" void fs_scan_prof_ptr(void **p) { cudaGetSymbolAddress(p, fs::fs_scan_prof); }
-namespace fs {
-#define FS_PROF_T(var) long long var = clock64()
-#define FS_PROF_ADD(slot, t0) \
-    if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[slot], (unsigned long long)(clock64() - (t0)))
-#else
-#define FS_PROF_T(var)
-#define FS_PROF_ADD(slot, t0)
-#endif
 
 // 16-byte vectors per lane per tile: 8 for 8-byte (value, flag) pairs, 4 for wider ones
 template <int OP, typename T> struct ScanShape {
@@ -416,582 +402,6 @@ scan_kernel(const T *__restrict__ in0, const float *__restrict__ in1, int64_t n,
         }
         __syncthreads();  // smem buffers, s_tile and s_ex reuse
     }
-}
-
-// ---------------------------------------------------------------- deferred look-back scan
-// Aggregates never wait; look-backs are deferred.  Iteration i of a CTA:
-//   A. claim tile t_i, TMA it from HBM, reduce it and publish its aggregate
-//      (no dependency on any other tile -> aggregates flow at read speed)
-//   C. for the tile t_{i-D} this CTA claimed D iterations ago: TMA it again
-//      (it is still in the 126 MB L2: D x #CTAs x 32 KB ~ 38 MB), scan it
-//      locally, look back (its predecessors published their aggregates about D
-//      iterations ago, so the look-back almost never spins), publish its
-//      inclusive prefix (helping forward) and write it.
-// HBM traffic stays one read + one write per element; the second read hits L2.
-template <int OP, typename T, bool SEG, int R, int D>
-__global__ void __launch_bounds__(kScanThreads, 768 / kScanThreads)
-scan_dl_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
-               int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
-               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanShape<OP, T>::PACK> ts, int64_t ntiles) {
-    using O = Op<OP, T>;
-    using SO = SOp<O, SEG>;
-    using S = typename SO::S;
-    constexpr int VEC = 16 / sizeof(T), NW = kScanThreads / 32;
-    constexpr int64_t TILE = (int64_t)kScanThreads * R * VEC;
-    constexpr unsigned TILE_BYTES = kScanThreads * R * 16;
-    constexpr int WIN = kScanThreads, RING = D + 2;
-    // buffers 0,1: new tiles (A, double-buffered); 2,3: deferred tiles (C, double-buffered)
-    extern __shared__ __align__(128) unsigned char sbuf[];
-    __shared__ uint64_t bars[4];
-    __shared__ int64_t s_ring[RING];
-    __shared__ S s_wtot[NW], s_wex[NW], s_ex, s_lb_tot[NW];
-    __shared__ __align__(16) int s_lb_min[NW];  // aligned: the min over it is read with 16-byte loads
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    // offset in its segment of this lane's first element of row q: one 64-bit modulo per
-    // tile, then steps of 32*VEC elements (rows of a lane's tile are 32*VEC apart)
-    const int64_t seg_step = SEG ? ((int64_t)32 * VEC) % L : 0;
-    int64_t seg_r0 = 0, seg_q0 = -1;
-    auto seg_off = [&](int64_t p0, int q) -> int64_t {
-        if (q == 0 || seg_q0 < 0) {
-            seg_r0 = p0 % L;
-        } else {
-            seg_r0 += seg_step;
-            if (seg_r0 >= L) seg_r0 -= L;
-        }
-        seg_q0 = q;
-        return seg_r0;
-    };
-    unsigned par = 0u;
-    auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
-    auto issue = [&](int b, int64_t t) {
-        if (t >= 0 && t < ntiles && full_tile(t)) {
-            fence_proxy_async();
-            mbar_expect_tx(&bars[b], TILE_BYTES);
-            tma_load_1d(sbuf + b * TILE_BYTES, in + t * TILE, TILE_BYTES, &bars[b]);
-        }
-    };
-    auto load_row = [&](int b, int64_t t, int q, T (&x)[VEC]) {
-        const int64_t p0 = t * TILE + (int64_t)warp * 32 * R * VEC + ((int64_t)q * 32 + lane) * VEC;
-        if (full_tile(t)) {
-            const Vec16<T> a =
-                *reinterpret_cast<const Vec16<T> *>(sbuf + b * TILE_BYTES + (((warp * R + q) * 32 + lane) << 4));
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) x[k] = a.e[k];
-        } else {
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) x[k] = p0 + k < n ? in[p0 + k] : T(0);
-        }
-        return p0;
-    };
-    auto lifted = [&](const T (&x)[VEC], int64_t p0, int k, int64_t &r) {
-        S e;
-        if (p0 + k < n) {
-            e.v = O::lift(x[k], SEG ? r : ibase + p0 + k);
-            e.f = SEG ? (r == 0) : 0;
-        } else {
-            e = SO::id();
-        }
-        if (SEG) {
-            ++r;
-            if (r == L) r = 0;
-        }
-        return e;
-    };
-    // ordered local scan of the tile in buffer b: per-row prefixes pre[], s_wex[], returns aggregate
-    auto local_scan = [&](int b, int64_t t, S (&pre)[R]) {
-        if (full_tile(t)) {
-            mbar_wait(&bars[b], (par >> b) & 1u);
-            par ^= 1u << b;
-        }
-        S carry_w = SO::id();
-#pragma unroll
-        for (int q = 0; q < R; ++q) {
-            T x[VEC];
-            const int64_t p0 = load_row(b, t, q, x);
-            int64_t r = SEG ? seg_off(p0, q) : 0;
-            S run = SO::id();
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) run = SO::comb(run, lifted(x, p0, k, r));
-            S a = run;
-#pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const S o = SO::up(a, off);
-                if (lane >= off) a = SO::comb(o, a);
-            }
-            S ex = SO::up(a, 1);
-            if (lane == 0) ex = SO::id();
-            pre[q] = SO::comb(carry_w, ex);
-            carry_w = SO::comb(carry_w, SO::bcast(a, 31));
-        }
-        if (lane == 0) s_wtot[warp] = carry_w;
-        __syncthreads();
-        S a = lane < NW ? s_wtot[lane] : SO::id();
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const S o = SO::up(a, off);
-            if (lane >= off) a = SO::comb(o, a);
-        }
-        S wex = SO::up(a, 1);
-        if (lane == 0) wex = SO::id();
-        if (warp == 0 && lane < NW) s_wex[lane] = wex;
-        const S agg = SO::bcast(a, NW - 1);
-        __syncthreads();
-        return agg;
-    };
-    // Aggregate of a tile for its look-back record, without scanning it: every table
-    // operator is commutative, so lanes fold their elements in any order and the CTA
-    // reduces; for the segmented operator only the elements at or after the tile's last
-    // segment start contribute, and that start is known in closed form (regular segments).
-    __shared__ typename O::V s_red[NW];
-    auto tile_aggregate = [&](int b, int64_t t) {
-        if (full_tile(t)) {
-            mbar_wait(&bars[b], (par >> b) & 1u);
-            par ^= 1u << b;
-        }
-        const int64_t t0 = t * TILE, t1 = (t + 1) * TILE < n ? (t + 1) * TILE : n;
-        int64_t keep = t0;
-        int flag = 0;
-        if (SEG) {
-            const int64_t last_start = ((t1 - 1) / L) * L;
-            flag = last_start >= t0;
-            keep = flag ? last_start : t0;
-        }
-        typename O::V acc = O::id();
-#pragma unroll
-        for (int q = 0; q < R; ++q) {
-            T x[VEC];
-            const int64_t p0 = load_row(b, t, q, x);
-            int64_t r = SEG ? seg_off(p0, q) : 0;
-#pragma unroll
-            for (int k = 0; k < VEC; ++k) {
-                const int64_t pk = p0 + k;
-                if (pk < t1 && pk >= keep) acc = O::comb(acc, O::lift(x[k], SEG ? r : ibase + pk));
-                if (SEG) {
-                    ++r;
-                    if (r == L) r = 0;
-                }
-            }
-        }
-        acc = group_reduce<O>(acc);
-        if (lane == 0) s_red[warp] = acc;
-        __syncthreads();
-        typename O::V tot = O::id();
-#pragma unroll
-        for (int q = 0; q < NW; ++q) tot = O::comb(tot, s_red[q]);
-        __syncthreads();
-        return S{tot, flag};
-    };
-    auto carry_in = [&]() {
-        S c0 = SO::id();
-        if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-        return c0;
-    };
-
-    S pre[R];
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int q = 0; q < 4; ++q) mbar_init(&bars[q], 1);
-        fence_mbar_init();
-        const int64_t t0 = (int64_t)atomicAdd(counter, 1u);
-        s_ring[0] = t0;
-        issue(0, t0);
-    }
-    for (int64_t i = 0;; ++i) {
-        if (threadIdx.x == 0) {
-            // prefetch for iteration i+1: claim t_{i+1} (stop claiming once past the end)
-            const int64_t cur = s_ring[i % RING];
-            const int64_t nxt = cur >= ntiles ? ntiles : (int64_t)atomicAdd(counter, 1u);
-            s_ring[(i + 1) % RING] = nxt;
-            issue((int)((i + 1) & 1), nxt);
-            issue(2 + (int)((i + 1) & 1), i + 1 >= D ? s_ring[(i + 1 - D) % RING] : -1);
-        }
-        __syncthreads();
-        const int64_t ti = s_ring[i % RING];
-        const int64_t told = i >= D ? s_ring[(i - D) % RING] : -1;
-        if (ti >= ntiles && (told < 0 || told >= ntiles)) {
-            bool more = false;
-            for (int64_t q = i - D + 1; q < i; ++q)
-                if (q >= 0 && s_ring[q % RING] < ntiles) more = true;
-            if (!more) break;
-        }
-        const int bA = (int)(i & 1), bC = 2 + (int)(i & 1);
-        FS_PROF_T(pa);
-        // A. aggregate of the new tile
-        if (ti < ntiles) {
-            const S agg = tile_aggregate(bA, ti);
-            if (threadIdx.x == 0) {
-                if (ti == 0) ts.publish(0, SO::comb(carry_in(), agg), kStIncl);
-                else ts.publish(ti, agg, kStAgg);
-            }
-        }
-        FS_PROF_ADD(1, pa);
-        FS_PROF_T(pc);
-        // C. scan + write the tile claimed D iterations ago
-        if (told >= 0 && told < ntiles) {
-            const S agg = local_scan(bC, told, pre);
-            FS_PROF_ADD(2, pc);
-            FS_PROF_T(pl);
-            S exc = SO::id();
-            if (told == 0) {
-                exc = carry_in();
-            } else {
-                int64_t j = told - 1;
-                for (int step = 0;; ++step) {
-                    const int64_t idx = j - threadIdx.x;
-                    const bool mine = idx >= 0;
-                    S v = SO::id();
-                    unsigned st = kStIncl;
-                    if (mine) {
-                        do {
-                            st = ts.poll(idx, v);
-                        } while (st == 0);
-                    }
-#ifdef FS_SCAN_PROFILE
-                    if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[5], 1ull);
-#endif
-                    const unsigned m = __ballot_sync(0xffffffffu, mine && st == kStIncl);
-                    if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 20;
-                    __syncthreads();
-                    int kk = 1 << 20;
-#pragma unroll
-                    for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
-                    if ((int)threadIdx.x > kk || !mine) v = SO::id();
-                    S a = v;
-#pragma unroll
-                    for (int off = 1; off < 32; off <<= 1) {
-                        const S o = SO::down(a, off);
-                        if (lane + off < 32) a = SO::comb(o, a);
-                    }
-                    if (lane == 0) s_lb_tot[warp] = a;
-                    __syncthreads();
-                    S left = SO::id();
-#pragma unroll
-                    for (int q = NW - 1; q > warp; --q) left = SO::comb(left, s_lb_tot[q]);
-                    S P = SO::id();
-#pragma unroll
-                    for (int q = NW - 1; q >= 0; --q) P = SO::comb(P, s_lb_tot[q]);
-                    if (step == 0 && kk < (1 << 20) && mine && (int)threadIdx.x < kk && st == kStAgg)
-                        ts.publish(idx, SO::comb(left, a), kStIncl);  // help forward
-                    exc = SO::comb(P, exc);
-                    __syncthreads();
-                    if (kk < (1 << 20) || exc.f) break;
-                    j -= WIN;
-                }
-                if (threadIdx.x == 0) ts.publish(told, SO::comb(exc, agg), kStIncl);
-            }
-            if (threadIdx.x == 0) s_ex = exc;
-            __syncthreads();
-            FS_PROF_ADD(3, pl);
-            FS_PROF_T(pw);
-            const S base = SO::comb(s_ex, s_wex[warp]);
-#pragma unroll
-            for (int q = 0; q < R; ++q) {
-                T x[VEC];
-                const int64_t p0 = load_row(bC, told, q, x);
-                S run = SO::comb(base, pre[q]);
-                int64_t r = SEG ? seg_off(p0, q) : 0;
-                T y[VEC];
-                int64_t yi[VEC];
-#pragma unroll
-                for (int k = 0; k < VEC; ++k) {
-                    run = SO::comb(run, lifted(x, p0, k, r));
-                    y[k] = O::val(run.v);
-                    yi[k] = O::idx(run.v);
-                }
-                if (p0 + VEC <= n) {
-                    Vec16<T> w;
-#pragma unroll
-                    for (int k = 0; k < VEC; ++k) w.e[k] = y[k];
-                    int4 wv;
-                    memcpy(&wv, &w, 16);
-                    *reinterpret_cast<int4 *>(out + p0) = wv;
-                } else {
-#pragma unroll
-                    for (int k = 0; k < VEC; ++k)
-                        if (p0 + k < n) out[p0 + k] = y[k];
-                }
-                if (OP == kArgmin) {
-#pragma unroll
-                    for (int k = 0; k < VEC; ++k)
-                        if (p0 + k < n) out_idx[p0 + k] = yi[k];
-                }
-            }
-            FS_PROF_ADD(4, pw);
-        }
-        __syncthreads();
-#ifdef FS_SCAN_PROFILE
-        if (threadIdx.x == 0) atomicAdd(&fs_scan_prof[0], 1ull);
-#endif
-    }
-}
-
-// ws body: [0,256) tile counter | status words (8 B per tile) | aggs | incls
-// ---------------------------------------------------------------- thread-contiguous TMA scan
-// The default path for 16-byte aligned inputs and outputs.  Every tile moves
-// HBM -> shared memory by one TMA bulk load and shared memory -> HBM by one TMA
-// bulk store; threads never touch global memory for a full tile.  Thread t owns
-// the R contiguous 16-byte vectors t*R .. t*R+R-1 of the tile (R odd: the eight
-// threads of a 16-byte shared-memory wavefront hit eight distinct bank groups),
-// so a tile costs one sequential fold per element, one warp scan and one block
-// scan of per-thread totals, and one (+) per element to apply the prefix, which
-// is written back in place and stored by TMA.  The ST-stage ring keeps ST-2
-// tiles of loads in flight per CTA while a tile is scanned and one is drained
-// by its bulk store; two CTAs per SM overlap one CTA's look-back wait with the
-// other's work.  Tiles are claimed in order from an atomic counter (forward
-// progress); the look-back window is the whole CTA.  For the segmented
-// operator a tile whose aggregate carries a segment start publishes it as its
-// inclusive prefix at once ((e, agg) = agg when agg.f, footnote 5's operator),
-// and a tile that starts a segment never looks back.
-#ifndef FS_SCANT_NT
-#define FS_SCANT_NT 256
-#endif
-#ifndef FS_SCANT_R
-#define FS_SCANT_R 3
-#endif
-#ifndef FS_SCANT_ST
-#define FS_SCANT_ST 5
-#endif
-#ifndef FS_SCANT_DYN
-#define FS_SCANT_DYN 0
-#endif
-#ifndef FS_SCANT_AHEAD
-#define FS_SCANT_AHEAD 1
-#endif
-#ifndef FS_SCANT_MINB
-#define FS_SCANT_MINB 3
-#endif
-constexpr int kScanTThreads = FS_SCANT_NT;
-template <int OP, typename T> struct ScanTShape {
-    static constexpr bool PACK = OP != kArgmin && sizeof(T) == 4;
-    static constexpr int R = PACK ? FS_SCANT_R : 3;
-    static_assert(R % 2 == 1, "R must be odd (bank-conflict-free thread-contiguous vectors)");
-    static constexpr int ST = FS_SCANT_ST;
-    static_assert(ST >= 3, "ring needs >= 3 stages (aggregates run one tile ahead of the scan)");
-    static constexpr int VEC = 16 / sizeof(T);
-    static constexpr int E = R * VEC;  // elements per thread per tile
-    static constexpr int64_t TILE = (int64_t)kScanTThreads * E;
-    static constexpr unsigned TILE_BYTES = kScanTThreads * R * 16;
-};
-
-template <int OP, typename T, bool SEG>
-__global__ void __launch_bounds__(kScanTThreads, FS_SCANT_MINB)
-scan_tc_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
-               int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
-               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanTShape<OP, T>::PACK> ts, int64_t ntiles) {
-    using O = Op<OP, T>;
-    using SO = SOp<O, SEG>;
-    using S = typename SO::S;
-    using Sh = ScanTShape<OP, T>;
-    constexpr int VEC = Sh::VEC, R = Sh::R, E = Sh::E, ST = Sh::ST, NW = kScanTThreads / 32;
-    constexpr int64_t TILE = Sh::TILE;
-    constexpr unsigned TB = Sh::TILE_BYTES;
-    extern __shared__ __align__(128) unsigned char sbuf[];
-    __shared__ uint64_t bars[ST];
-    __shared__ int64_t s_tile[ST];
-    __shared__ S s_wtot[NW], s_lb_val[NW];
-    __shared__ int s_lb_min[NW];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    auto full_tile = [&](int64_t t) { return (t + 1) * TILE <= n; };
-    // static round-robin tiles: iteration `it` of this CTA scans tile blockIdx.x + it * gridDim.x
-    // (grid <= resident CTAs, so every tile is owned by a running CTA that visits its
-    // tiles in increasing order: forward progress)
-    auto tile_of = [&](int it) {
-        return FS_SCANT_DYN ? s_tile[it % ST] : (int64_t)blockIdx.x + (int64_t)it * gridDim.x;
-    };
-    auto issue = [&](int it) {  // thread 0 only
-        const int s = it % ST;
-        if (FS_SCANT_DYN) s_tile[s] = (int64_t)atomicAdd(counter, 1u);
-        const int64_t t = tile_of(it);
-        if (t < ntiles && full_tile(t)) {
-            fence_proxy_async();
-            mbar_expect_tx(&bars[s], TB);
-            tma_load_1d(sbuf + s * TB, in + t * TILE, TB, &bars[s]);
-        }
-    };
-
-    // per-tile state carried from phase A (aggregate, one iteration ahead) to phase C
-    struct Pre {
-        S tex, wex, agg;
-    };
-    auto load_x = [&](int s, int64_t tile, bool full, int64_t e0, T (&x)[E]) {
-        if (full) {
-            const unsigned char *sv = sbuf + s * TB + threadIdx.x * (R * 16);
-#pragma unroll
-            for (int j = 0; j < R; ++j) {
-                const Vec16<T> a = *reinterpret_cast<const Vec16<T> *>(sv + j * 16);
-#pragma unroll
-                for (int k = 0; k < VEC; ++k) x[j * VEC + k] = a.e[k];
-            }
-        } else {
-#pragma unroll
-            for (int i = 0; i < E; ++i) x[i] = e0 + i < n ? in[e0 + i] : T(0);
-        }
-    };
-    auto lifted = [&](const T (&x)[E], bool full, int64_t e0, int i, int64_t &r) {
-        S e;
-        if (full || e0 + i < n) {
-            e.v = O::lift(x[i], SEG ? r : ibase + e0 + i);
-            e.f = SEG ? (r == 0) : 0;
-        } else {
-            e = SO::id();
-        }
-        if (SEG) {
-            ++r;
-            if (r == L) r = 0;
-        }
-        return e;
-    };
-    // phase A of iteration `it`: wait for the tile, fold, warp + block scan of thread
-    // totals, publish the aggregate (or the inclusive prefix when it needs no look-back)
-    auto phase_a = [&](int it, Pre &p) {
-        const int s = it % ST;
-        const int64_t tile = tile_of(it);
-        const bool full = full_tile(tile);
-        const int64_t e0 = tile * TILE + (int64_t)threadIdx.x * E;
-        if (full) mbar_wait(&bars[s], (unsigned)(it / ST) & 1u);
-        T x[E];
-        load_x(s, tile, full, e0, x);
-        S tot = SO::id();
-        int64_t r = SEG ? e0 % L : 0;
-#pragma unroll
-        for (int i = 0; i < E; ++i) tot = SO::comb(tot, lifted(x, full, e0, i, r));
-        S a = tot;
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const S o = SO::up(a, off);
-            if (lane >= off) a = SO::comb(o, a);
-        }
-        p.tex = SO::up(a, 1);
-        if (lane == 0) p.tex = SO::id();
-        if (lane == 31) s_wtot[warp] = a;
-        __syncthreads();
-        S b = lane < NW ? s_wtot[lane] : SO::id();
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const S o = SO::up(b, off);
-            if (lane >= off) b = SO::comb(o, b);
-        }
-        S bex = SO::up(b, 1);
-        if (lane == 0) bex = SO::id();
-        p.wex = SO::bcast(bex, warp);
-        p.agg = SO::bcast(b, NW - 1);
-        if (threadIdx.x == 0) {
-            if (tile == 0) {
-                S c0 = SO::id();
-                if (carry) c0 = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-                ts.publish(0, SO::comb(c0, p.agg), kStIncl);
-            } else {
-                // a flagged aggregate is already the inclusive prefix
-                ts.publish(tile, p.agg, (SEG && p.agg.f) ? kStIncl : kStAgg);
-            }
-        }
-    };
-
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int s = 0; s < ST; ++s) mbar_init(&bars[s], 1);
-        fence_mbar_init();
-#pragma unroll
-        for (int q = 0; q < ST - 1; ++q) issue(q);
-    }
-    __syncthreads();
-    Pre cur, nxt;
-    if (FS_SCANT_AHEAD && tile_of(0) < ntiles) phase_a(0, cur);
-    for (int it = 0;; ++it) {
-        const int s = it % ST;
-        const int64_t tile = tile_of(it);
-        if (tile >= ntiles) break;
-        const bool full = full_tile(tile);
-        const int64_t e0 = tile * TILE + (int64_t)threadIdx.x * E;
-        // aggregate of the next tile first: it never waits on anything but its own data
-        if (!FS_SCANT_AHEAD) phase_a(it, cur);
-        else if (tile_of(it + 1) < ntiles) phase_a(it + 1, nxt);
-        // ---- look-back for this tile (its predecessors published at least an iteration ago)
-        S exc = SO::id();
-        if (tile == 0) {
-            if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
-        } else if (!(SEG && (tile * TILE) % L == 0)) {
-            int64_t j = tile - 1;
-            while (true) {
-                const int64_t idx = j - threadIdx.x;
-                S v = SO::id();
-                unsigned st = kStIncl;
-                if (idx >= 0) {
-                    do {
-                        st = ts.poll(idx, v);
-                    } while (st == 0);
-                }
-                const unsigned m = __ballot_sync(0xffffffffu, idx >= 0 && st == kStIncl);
-                if (lane == 0) s_lb_min[warp] = m ? warp * 32 + __ffs(m) - 1 : 1 << 30;
-                __syncthreads();
-                int kk = 1 << 30;
-#pragma unroll
-                for (int q = 0; q < NW; ++q) kk = min(kk, s_lb_min[q]);
-                if ((int)threadIdx.x > kk || idx < 0) v = SO::id();
-                S w = v;
-#pragma unroll
-                for (int off = 1; off < 32; off <<= 1) {
-                    const S o = SO::down(w, off);
-                    if (lane + off < 32) w = SO::comb(o, w);
-                }
-                if (lane == 0) s_lb_val[warp] = w;
-                __syncthreads();
-                S P = SO::id(), left = SO::id();
-#pragma unroll
-                for (int q = NW - 1; q >= 0; --q) {
-                    if (q > warp) left = SO::comb(left, s_lb_val[q]);
-                    P = SO::comb(P, s_lb_val[q]);
-                }
-                // help forward: a predecessor found as an aggregate between this tile and the
-                // nearest inclusive prefix gets its inclusive prefix published now
-                if (kk < (1 << 30) && idx >= 0 && (int)threadIdx.x < kk && st == kStAgg)
-                    ts.publish(idx, SO::comb(left, w), kStIncl);
-                exc = SO::comb(P, exc);
-                __syncthreads();  // s_lb_* reuse
-                if (kk < (1 << 30) || exc.f || j < kScanTThreads) break;
-                j -= kScanTThreads;
-            }
-            if (threadIdx.x == 0 && !(SEG && cur.agg.f)) ts.publish(tile, SO::comb(exc, cur.agg), kStIncl);
-        }
-        // ---- phase C: apply the prefix; full tiles go back in place and out by one bulk store
-        {
-            T x[E];
-            load_x(s, tile, full, e0, x);
-            S run = SO::comb(exc, SO::comb(cur.wex, cur.tex));
-            int64_t r = SEG ? e0 % L : 0;
-            T y[E];
-#pragma unroll
-            for (int i = 0; i < E; ++i) {
-                run = SO::comb(run, lifted(x, full, e0, i, r));
-                y[i] = O::val(run.v);
-                if (OP == kArgmin && (full || e0 + i < n)) out_idx[e0 + i] = O::idx(run.v);
-            }
-            if (full) {
-                unsigned char *sv = sbuf + s * TB + threadIdx.x * (R * 16);
-#pragma unroll
-                for (int j = 0; j < R; ++j) {
-                    Vec16<T> w;
-#pragma unroll
-                    for (int k = 0; k < VEC; ++k) w.e[k] = y[j * VEC + k];
-                    *reinterpret_cast<Vec16<T> *>(sv + j * 16) = w;
-                }
-                fence_proxy_async();  // generic-proxy smem writes -> visible to the bulk store
-            } else {
-#pragma unroll
-                for (int i = 0; i < E; ++i)
-                    if (e0 + i < n) out[e0 + i] = y[i];
-            }
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            if (full) tma_store_1d(out + tile * TILE, sbuf + s * TB, TB);
-            bulk_commit();
-            bulk_wait_read<1>();  // the store of stage (it-1)%ST has read its smem
-            issue(it + ST - 1);
-        }
-        if (FS_SCANT_AHEAD) cur = nxt;
-    }
-    if (threadIdx.x == 0) bulk_wait<0>();
 }
 
 // ---------------------------------------------------------------- warp-specialised slab scan
@@ -1597,8 +1007,7 @@ template <int OP, typename T> struct ScanRun {
             ts.incls = ts.aggs + ntiles;
         }
         if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntiles), st) != cudaSuccess) return FS_ERR_CUDA;
-        if constexpr (TMA && !NN) {
-#ifndef FS_SCAN_TC
+        if constexpr (TMA && !NN) {  // the warp-specialised slab scan (16-byte aligned buffers)
             {
                 using ShW = ScanWShape<OP, T>;
                 const int64_t ntw = ceil_div(n, ShW::TILE);
@@ -1613,30 +1022,6 @@ template <int OP, typename T> struct ScanRun {
                                                                   (const T *)carry, carry_idx, ts, ntw, (int)tps);
                 return launch_status();
             }
-#endif
-#ifndef FS_SCAN_DEFERRED
-            using ShB = ScanTShape<OP, T>;
-            const int64_t ntb = ceil_div(n, ShB::TILE);
-            auto kb = scan_tc_kernel<OP, T, SEG>;
-            const int smemb = ShB::ST * (int)ShB::TILE_BYTES;
-            cudaFuncSetAttribute((const void *)kb, cudaFuncAttributeMaxDynamicSharedMemorySize, smemb);
-            const int64_t capb = resident_blocks((const void *)kb, kScanTThreads, smemb);
-            const int64_t gridb = ntb < capb ? ntb : capb;
-            kb<<<(unsigned)gridb, kScanTThreads, smemb, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
-                                                               (const T *)carry, carry_idx, counter, ts, ntb);
-            return launch_status();
-#endif
-            // same tile shape as the ws sizing (Sh::R rows of 16-byte vectors per thread)
-            // deferred look-back, 4 buffers of half-size tiles (same tile grid as the ws sizing)
-            // D = 3 iterations of deferral (swept 1..3 and R = 4/8 on B200: R4 D3 fastest)
-            auto kp = scan_dl_kernel<OP, T, SEG, Sh::R, 3>;
-            const int smem = 4 * (int)Sh::TILE_BYTES;
-            cudaFuncSetAttribute((const void *)kp, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            const int64_t cap = resident_blocks((const void *)kp, kScanThreads, smem);
-            const int64_t grid = ntiles < cap ? ntiles : cap;
-            kp<<<(unsigned)grid, kScanThreads, smem, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
-                                                           (const T *)carry, carry_idx, counter, ts, ntiles);
-            return launch_status();
         }
         auto k = scan_kernel<OP, T, NN, SEG, TMA>;
         const int smem = TMA ? 2 * (int)Sh::TILE_BYTES : 0;
@@ -1904,32 +1289,32 @@ colscan_narrow_kernel(const T *__restrict__ x, int64_t m, int64_t w, int WV, int
         const bool ok = r < r1;
         Vec16<T> e;
         if (ok) e = as_vec<T>(ldg16(x + r * w + cv * VEC));
-        if (!SCAN) {
+        if constexpr (!SCAN) {
             if (ok)
 #pragma unroll
                 for (int k = 0; k < VEC; ++k) acc[k] = O::comb(acc[k], O::lift(e.e[k], r));
-            continue;
-        }
-        V v[VEC];
+        } else {
+            V v[VEC];
 #pragma unroll
-        for (int k = 0; k < VEC; ++k) v[k] = ok ? O::lift(e.e[k], r) : O::id();
+            for (int k = 0; k < VEC; ++k) v[k] = ok ? O::lift(e.e[k], r) : O::id();
 #pragma unroll 1
-        for (int dd = 1; dd < RPW; dd <<= 1) {
+            for (int dd = 1; dd < RPW; dd <<= 1) {
+#pragma unroll
+                for (int k = 0; k < VEC; ++k) {
+                    const V o = shfl_up(v[k], dd * WV);
+                    if (ro >= dd) v[k] = O::comb(o, v[k]);
+                }
+            }
+            Vec16<T> o;
 #pragma unroll
             for (int k = 0; k < VEC; ++k) {
-                const V o = shfl_up(v[k], dd * WV);
-                if (ro >= dd) v[k] = O::comb(o, v[k]);
+                const V z = O::comb(acc[k], v[k]);
+                o.e[k] = O::val(z);
+                if (ok && OP == kArgmin) out_idx[r * w + cv * VEC + k] = O::idx(z);
+                acc[k] = shfl_idx(z, (RPW - 1) * WV + cv);  // carry = the step's last row of this column
             }
+            if (ok) *reinterpret_cast<int4 *>(out + r * w + cv * VEC) = *reinterpret_cast<const int4 *>(&o);
         }
-        Vec16<T> o;
-#pragma unroll
-        for (int k = 0; k < VEC; ++k) {
-            const V z = O::comb(acc[k], v[k]);
-            o.e[k] = O::val(z);
-            if (ok && OP == kArgmin) out_idx[r * w + cv * VEC + k] = O::idx(z);
-            acc[k] = shfl_idx(z, (RPW - 1) * WV + cv);  // carry = the step's last row of this column
-        }
-        if (ok) *reinterpret_cast<int4 *>(out + r * w + cv * VEC) = *reinterpret_cast<const int4 *>(&o);
     }
     if (!SCAN) {
         for (int dd = WV; dd < 32; dd <<= 1)
