@@ -488,6 +488,19 @@ def test_seg_scan_col_narrow(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan col narrow {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("seglen", [4, 64, 512])
+def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
+    """KS0 needs 16-byte aligned buffers: a misaligned view takes the look-back scan and
+    still matches the oracle."""
+    nseg = 777
+    for dt, op in ((np.float32, "add"), (np.int32, "max"), (np.float32, "argmin")):
+        x = workloads.mixed(nseg * seglen, seglen, dt)
+        got = fs.seg_scan(cu(x, 1), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan misaligned {seglen} {op}")
+
+
 def test_seg_scan_misaligned(fs):
     x = workloads.mixed(50 * 999, 4, np.int64)
     got = fs.seg_scan(cu(x, 1), 50, 999, "add")
