@@ -376,17 +376,37 @@ kmeans_step_kernel(const float *__restrict__ pts, int64_t n, int d, const float 
     __syncthreads();
     if (!last) return;
     const int G = gridDim.x;
+    // four interleaved accumulators (a fixed order): ~32 independent L2 loads in flight
     for (int cc = threadIdx.x; cc < k; cc += kKmThreads) {
-        unsigned a = 0;
-        for (int q = 0; q < G; ++q) a += (unsigned)__ldcg(pcounts + (int64_t)q * k + cc);
+        unsigned a0 = 0, a1 = 0, a2 = 0, a3 = 0;
+        int q = 0;
+#pragma unroll 8
+        for (; q + 4 <= G; q += 4) {
+            const int *p = pcounts + (int64_t)q * k + cc;
+            a0 += (unsigned)__ldcg(p);
+            a1 += (unsigned)__ldcg(p + k);
+            a2 += (unsigned)__ldcg(p + 2 * k);
+            a3 += (unsigned)__ldcg(p + 3 * k);
+        }
+        for (; q < G; ++q) a0 += (unsigned)__ldcg(pcounts + (int64_t)q * k + cc);
+        const unsigned a = a0 + a1 + a2 + a3;
         s_cnt[cc] = (int)a;
         counts[cc] = (int32_t)a;
     }
     __syncthreads();
     for (int64_t e = threadIdx.x; e < kd; e += kKmThreads) {
-        float a = 0.f;
+        float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+        int q = 0;
 #pragma unroll 8
-        for (int q = 0; q < G; ++q) a = __fadd_rn(a, __ldcg(partials + (int64_t)q * kd + e));
+        for (; q + 4 <= G; q += 4) {
+            const float *p = partials + (int64_t)q * kd + e;
+            a0 = __fadd_rn(a0, __ldcg(p));
+            a1 = __fadd_rn(a1, __ldcg(p + kd));
+            a2 = __fadd_rn(a2, __ldcg(p + 2 * kd));
+            a3 = __fadd_rn(a3, __ldcg(p + 3 * kd));
+        }
+        for (; q < G; ++q) a0 = __fadd_rn(a0, __ldcg(partials + (int64_t)q * kd + e));
+        const float a = __fadd_rn(__fadd_rn(a0, a1), __fadd_rn(a2, a3));
         sums[e] = a;
         const int cc = (int)(e / d);
         if (new_cen) new_cen[e] = s_cnt[cc] > 0 ? __fdiv_rn(a, (float)s_cnt[cc]) : cen[e];
