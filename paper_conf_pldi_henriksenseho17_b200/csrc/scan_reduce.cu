@@ -178,9 +178,15 @@ scan_reduce_kernel(const T *__restrict__ x, int64_t n, int64_t tiles_per_warp, S
     const int64_t W = (int64_t)gridDim.x * 8;
     const int64_t per = (W + 255) / 256;
     SRPair<C> q = FC::id();
-    for (int64_t w = threadIdx.x * per; w < min(W, (threadIdx.x + 1) * per); ++w) {
-        const SRPair<T> pw = ld_cg_pair(wparts + w);
-        q = FC::comb(q, SRPair<C>{(C)pw.A, (C)pw.R, pw.L});
+    const int64_t w0 = threadIdx.x * per, w1 = min(W, (threadIdx.x + 1) * per);
+    for (int64_t w = w0; w < w1; w += 8) {  // 8 loads in flight, then the ordered folds
+        SRPair<T> pw[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+            if (w + i < w1) pw[i] = ld_cg_pair(wparts + w + i);
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+            if (w + i < w1) q = FC::comb(q, SRPair<C>{(C)pw[i].A, (C)pw[i].R, pw[i].L});
     }
     __shared__ SRPair<C> sq[256];
     sq[threadIdx.x] = q;
