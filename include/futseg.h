@@ -287,6 +287,9 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       256 * 16/sizeof(elem), FS_ROW_MAJOR, 16-byte aligned buffers; others take 5):
  *       in-register scan, shuffle scan across the lanes of a segment and, for rows
  *       longer than a warp's 32 vectors, a shared-memory combine across its warps
+ *   8 = KS1 fs_seg_scan of short rows that are not powers of two (seglen <= 32,
+ *       FS_ROW_MAJOR, 16-byte aligned, op != ARGMIN): 256 rows staged through shared
+ *       memory, a thread scans a row
  * Returns -1 for invalid arguments. */
 int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen,
                       int32_t layout);

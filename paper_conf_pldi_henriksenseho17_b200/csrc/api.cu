@@ -510,7 +510,9 @@ int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t 
     if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1) return 4;
     if (prim_is_scan) {
         const int64_t vec = 16 / (int64_t)dtype_size(op.dtype);
-        return (nseg > 1 && (seglen & (seglen - 1)) == 0 && seglen <= 256 * vec) ? 7 : 5;
+        if (nseg > 1 && (seglen & (seglen - 1)) == 0 && seglen <= 256 * vec) return 7;
+        if (nseg > 1 && seglen >= 2 && seglen <= 32 && op.op != FS_ARGMIN) return 8;
+        return 5;
     }
     return seg_reduce_regime(op.op, op.dtype, nseg, seglen);
 }

@@ -990,6 +990,55 @@ segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ ou
     }
 }
 
+// KS1: short rows of any length L <= 32 that are not powers of two (a 16-byte vector then
+// straddles rows): a CTA stages 256 whole rows through shared memory with coalesced 16-byte
+// loads (index padded every 32 elements), thread t scans row t sequentially in place, and
+// the tile leaves with coalesced 16-byte stores.  No look-back, no per-element flags.
+template <int OP, typename T>
+__global__ void __launch_bounds__(256)
+segscan_tile_kernel(const T *__restrict__ x, int64_t nseg, int L, T *__restrict__ out) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T);
+    extern __shared__ __align__(16) unsigned char tsm[];
+    T *sm = reinterpret_cast<T *>(tsm);
+    auto pad = [](int i) { return i + (i >> 5); };
+    const int t = threadIdx.x;
+    const int64_t ntile = (nseg + 255) / 256;
+    for (int64_t tile = blockIdx.x; tile < ntile; tile += gridDim.x) {
+        const int64_t s0 = tile * 256;
+        const int rows = (int)min((int64_t)256, nseg - s0);
+        const int te = rows * L;                  // elements of the tile
+        const T *src = x + s0 * L;                // 16-byte aligned: 256 * L * sizeof(T) per tile
+        const int nv = te / VEC;
+        for (int v = t; v < nv; v += 256) {
+            const Vec16<T> e = as_vec<T>(ldg16(src + (int64_t)v * VEC));
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) sm[pad(v * VEC + k)] = e.e[k];
+        }
+        for (int i = nv * VEC + t; i < te; i += 256) sm[pad(i)] = src[i];
+        __syncthreads();
+        if (t < rows) {
+            V a = O::id();
+            for (int j = 0; j < L; ++j) {
+                const int i = pad(t * L + j);
+                a = j == 0 ? O::lift(sm[i], 0) : O::fold(a, sm[i], j);
+                sm[i] = O::val(a);
+            }
+        }
+        __syncthreads();
+        T *dst = out + s0 * L;
+        for (int v = t; v < nv; v += 256) {
+            Vec16<T> o;
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) o.e[k] = sm[pad(v * VEC + k)];
+            *reinterpret_cast<int4 *>(dst + (int64_t)v * VEC) = *reinterpret_cast<const int4 *>(&o);
+        }
+        for (int i = nv * VEC + t; i < te; i += 256) dst[i] = sm[pad(i)];
+        __syncthreads();
+    }
+}
+
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1069,6 +1118,20 @@ template <int OP, typename T> struct ScanRun {
                 grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
                 return launch_status();
+            }
+            if constexpr (OP != kArgmin) {  // (argmin's index output keeps the look-back path)
+                if (al && !carry && map->ibase == 0 && L >= 2 && L <= 32) {
+                    auto kt = segscan_tile_kernel<OP, T>;
+                    const int smem = (int)((256 * L + 256 * L / 32 + 1) * sizeof(T));
+                    if (smem > 48 * 1024)
+                        cudaFuncSetAttribute((const void *)kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                    const int64_t nseg = n / L;
+                    int64_t grid = ceil_div(nseg, 256);
+                    const int64_t cap = resident_blocks((const void *)kt, 256, (size_t)smem);
+                    grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
+                    kt<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, nseg, (int)L, (T *)out);
+                    return launch_status();
+                }
             }
             if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
             return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);

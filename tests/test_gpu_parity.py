@@ -501,6 +501,20 @@ def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
         assert_reduced(got, want, op, asum, f"segscan misaligned {seglen} {op}")
 
 
+@pytest.mark.parametrize("seglen", [3, 5, 7, 9, 12, 17, 31])
+@pytest.mark.parametrize("nseg", [1, 2, 255, 256, 257, 100_001])
+def test_seg_scan_short_rows_tile(fs, nseg, seglen):
+    """KS1 (regime 8): short non-power-of-two rows staged through shared memory (tiles of 256
+    rows, a ragged last tile, scalar tails of the vector loads); add/min/max on every dtype."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int32, "max"), (np.int64, "add")):
+        x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
+            workloads.mixed(nseg * seglen, nseg + seglen, dt)
+        got = fs.seg_scan(cu(x), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan tile {nseg}x{seglen} {dt.__name__} {op}")
+
+
 def test_seg_scan_misaligned(fs):
     x = workloads.mixed(50 * 999, 4, np.int64)
     got = fs.seg_scan(cu(x, 1), 50, 999, "add")
