@@ -55,5 +55,17 @@ pts, _ = workloads.c3_kmeans(n=20_011, d=34, k=32)
 fs.kmeans_step(cu(pts), cu(pts[:32].copy()), prev=cu(workloads.ints(20_011, 3, 0, 32)))
 pts, _ = workloads.c3_kmeans(n=5_003, d=7, k=5)
 fs.kmeans_step(cu(pts), cu(pts[:5].copy()))
+# seg_scan KS1 (short non-power-of-two rows), scan_reduce, seg_map_reduce (all regimes)
+for nseg, L in ((1001, 3), (257, 7), (300, 31)):
+    fs.seg_scan(x[: nseg * L], nseg, L, "add")
+    fs.seg_scan(xi[: nseg * L], nseg, L, "max")
+for red in ("add", "max", "min"):
+    fs.scan_reduce(x[:200_001], red)
+    fs.scan_reduce(xi[:77_777], red)
+for nseg, L in ((1000, 8), (300, 33), (5, 20_000)):
+    fs.seg_map_reduce(x[: nseg * L], nseg, L, 1.0, "add")
+    fs.seg_map_reduce(xi[: nseg * L], nseg, L, 2, "argmin")
+xb = cu(workloads.mixed(600 * 8192, 8, np.float32))  # CTA-per-row regime (>= 4 rows per SM)
+fs.seg_map_reduce(xb, 600, 8192, 1.0, "max")
 torch.cuda.synchronize()
 print("sanitize cases done")
