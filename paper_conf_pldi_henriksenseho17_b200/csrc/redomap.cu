@@ -61,20 +61,25 @@ __global__ void __launch_bounds__(NT) redomap_id_kernel(const T *__restrict__ x,
 
     V acc = O::id();
     if (gid < head) acc = O::fold(acc, x[gid], gid);
-    int64_t v = gid;
-    for (; v + (U - 1) * stride < nvec; v += U * stride) {
+    // a warp reads U consecutive 512-byte runs (one contiguous 2 KB block) per iteration and
+    // the warps stride over the array by blocks; every thread's indices still increase
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = gid >> 5, nw = stride >> 5;
+    const int64_t nblk = nvec / (32 * U);  // whole blocks
+    for (int64_t bk = gw; bk < nblk; bk += nw) {
+        const int64_t v0 = bk * 32 * U + lane;
         int4 r[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) r[u] = ldg16(xv + v + u * stride);
+        for (int u = 0; u < U; ++u) r[u] = ldg16(xv + v0 + u * 32);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const Vec16<T> e = as_vec<T>(r[u]);
-            const int64_t base = head + (v + u * stride) * VEC;
+            const int64_t base = head + (v0 + u * 32) * VEC;
 #pragma unroll
             for (int k = 0; k < VEC; ++k) acc = O::fold(acc, e.e[k], base + k);
         }
     }
-    for (; v < nvec; v += stride) {
+    for (int64_t v = nblk * 32 * U + gid; v < nvec; v += stride) {  // vectors past the last block
         const Vec16<T> e = as_vec<T>(ldg16(xv + v));
         const int64_t base = head + v * VEC;
 #pragma unroll
