@@ -164,6 +164,7 @@ __global__ void vadd_combine_kernel(const T *__restrict__ parts, int64_t P, int6
 
 // ------------------------------------------------------------------ host side
 constexpr int kRedU = 4;
+constexpr int kNnU = 2;
 
 template <int OP, typename T> struct RedomapId {
     static const void *kernel() { return (const void *)redomap_id_kernel<OP, T, kRedThreads, kRedU>; }
@@ -187,11 +188,12 @@ template <int OP, typename T> struct RedomapNN {
                          int64_t *out_idx, int64_t ibase, void *ws, cudaStream_t st) {
         using V = typename Op<OP, float>::V;
         const bool vect = (((uintptr_t)lat ^ (uintptr_t)lng) & 15) == 0;
-        const void *k = vect ? (const void *)redomap_nn_kernel<OP, kRedThreads, kRedU, true>
-                             : (const void *)redomap_nn_kernel<OP, kRedThreads, kRedU, false>;
+        const void *k = vect ? (const void *)redomap_nn_kernel<OP, kRedThreads, kNnU, true>
+                             : (const void *)redomap_nn_kernel<OP, kRedThreads, kNnU, false>;
         // the distance map costs ~40 instructions per record: spread small inputs (NN's
-        // 855,280 records) over the whole machine, one 4-record vector per thread minimum
-        const int64_t per_cta = (int64_t)kRedThreads * 4;
+        // 855,280 records) over the whole machine, kNnU 4-record vectors per thread, all of
+        // them loaded before the first is folded (one DRAM round trip, not kNnU)
+        const int64_t per_cta = (int64_t)kRedThreads * 4 * kNnU;
         int64_t grid = ceil_div(n, per_cta);
         grid = grid < 1 ? 1 : grid;
         const int64_t cap = resident_blocks(k, kRedThreads);
@@ -200,10 +202,10 @@ template <int OP, typename T> struct RedomapNN {
         V *parts = (V *)(w + kWsHeader);
         unsigned *ticket = (unsigned *)(w + kWsTicket);
         if (vect)
-            redomap_nn_kernel<OP, kRedThreads, kRedU, true>
+            redomap_nn_kernel<OP, kRedThreads, kNnU, true>
                 <<<(unsigned)grid, kRedThreads, 0, st>>>(lat, lng, n, q0, q1, parts, ticket, (float *)out, out_idx, ibase);
         else
-            redomap_nn_kernel<OP, kRedThreads, kRedU, false>
+            redomap_nn_kernel<OP, kRedThreads, kNnU, false>
                 <<<(unsigned)grid, kRedThreads, 0, st>>>(lat, lng, n, q0, q1, parts, ticket, (float *)out, out_idx, ibase);
         return launch_status();
     }
