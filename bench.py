@@ -189,17 +189,18 @@ def make_step(fs, W, world):
 # ------------------------------------------------------------------ SURVEY 8(f) "next" rows
 def time_next_rows(fs, W, dev, K, peak):
     """Each NEXT row timed on its own (one warm-up call, then CUDA events over K reps, L2
-    flushed before every rep by a 1 GB write outside the events; median and min reported).
+    flushed before every rep by READING a 1 GB buffer outside the events -- a write flush
+    would leave ~126 MB of dirty lines for the timed kernel to write back; median and min).
     Not part of the step value (8(a) rows only)."""
     import torch
-    flush = torch.empty(1 << 30, dtype=torch.uint8, device=dev)  # ~150 us of GPU time: the host stays ahead
+    flush = torch.ones(1 << 28, dtype=torch.float32, device=dev)  # 1 GB: ~160 us of reads, the host stays ahead
     rows = {}
 
     def timed(fn, reps=K):
         fn()  # warm-up: workspace growth, function attributes
         ms = []
         for _ in range(reps):
-            flush.zero_()
+            torch.amax(flush)  # evict by READING 1 GB: no dirty lines left to write back
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record()
             fn()

@@ -13,7 +13,7 @@ import paper_conf_pldi_henriksenseho17_b200 as fs  # noqa: E402
 pts, mem = workloads.c3_kmeans(keys="clustered")
 P, M = torch.from_numpy(pts).cuda(), torch.from_numpy(mem).cuda()
 cen = P[:5].clone()
-flush = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+flush = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
 b_sr = pts.shape[0] * (34 * 4 + 4)
 
 
@@ -22,7 +22,7 @@ def t(fn, cold, reps=20):
     ms = []
     for _ in range(reps):
         if cold:
-            flush.zero_()
+            torch.amax(flush)  # evict by READING 1 GB: no dirty lines left to write back
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
         fn()
