@@ -290,6 +290,10 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *   8 = KS1 fs_seg_scan of short rows that are not powers of two (seglen <= 32,
  *       FS_ROW_MAJOR, 16-byte aligned, op != ARGMIN): 256 rows staged through shared
  *       memory, a thread scans a row
+ *   9 = KS2 fs_seg_scan of long rows (at least 4 chunks of 256 x R vectors: 12288 f32,
+ *       4096 f32 argmin, 2048 8-byte elements) when there are at least
+ *       4 rows per SM (FS_ROW_MAJOR, in/out with the same 16-byte phase): a CTA owns
+ *       whole rows and scans them chunk by chunk with a running carry (no look-back)
  * Returns -1 for invalid arguments. */
 int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen,
                       int32_t layout);

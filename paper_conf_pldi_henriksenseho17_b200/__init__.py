@@ -44,7 +44,8 @@ LAYOUTS = {"row": 0, "col": 1}
 _DT = {torch.int32: FS_I32, torch.int64: FS_I64, torch.float32: FS_F32}
 REGIMES = {0: "KG1 smem tile", 1: "KG2 warp/segment", 2: "KG3 block/segment", 3: "KG4 multi-block/segment",
            4: "column (col-major)", 5: "segmented look-back scan", 6: "empty",
-           7: "KS0 short power-of-two scan (register + shuffle)", 8: "KS1 short-row scan (shared-memory tile)"}
+           7: "KS0 short power-of-two scan (register + shuffle)", 8: "KS1 short-row scan (shared-memory tile)",
+           9: "KS2 CTA-per-row scan with a running carry"}
 
 
 class fs_opdesc(ctypes.Structure):

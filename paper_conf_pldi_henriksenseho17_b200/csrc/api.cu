@@ -512,6 +512,8 @@ int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t 
         const int64_t vec = 16 / (int64_t)dtype_size(op.dtype);
         if (nseg > 1 && (seglen & (seglen - 1)) == 0 && seglen <= 256 * vec) return 7;
         if (nseg > 1 && seglen >= 2 && seglen <= 32 && op.op != FS_ARGMIN) return 8;
+        const int64_t ks2ch = 256 * vec * ((dtype_size(op.dtype) == 4 && op.op != FS_ARGMIN) ? 3 : 1);
+        if (seglen >= 4 * ks2ch && nseg >= 4 * (int64_t)sm_count()) return 9;
         return 5;
     }
     return seg_reduce_regime(op.op, op.dtype, nseg, seglen);

@@ -1039,6 +1039,136 @@ segscan_tile_kernel(const T *__restrict__ x, int64_t nseg, int L, T *__restrict_
     }
 }
 
+// KS2: rows long enough that a CTA should own whole rows (L > 256 vectors) and numerous
+// enough to fill the machine: a CTA scans its rows chunk by chunk with a running carry, so
+// rows never wait on other CTAs (no look-back).  A chunk is 256 threads x R contiguous
+// 16-byte vectors (thread-contiguous, R odd: conflict-free staging is not needed, the
+// vectors stay in registers); the next chunk's loads are in flight while this one is
+// scanned.  A misaligned row start is handled by a scalar head (thread 0), the ragged end
+// by a scalar tail.
+template <int OP, typename T, int R>
+__global__ void __launch_bounds__(256)
+segscan_cta_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int VEC = 16 / sizeof(T), E = R * VEC;
+    constexpr int64_t CH = 256 * (int64_t)E;  // elements per chunk
+    __shared__ V s_w[8];
+    __shared__ V s_carry;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    for (int64_t s = blockIdx.x; s < nseg; s += gridDim.x) {
+        const T *p = x + s * L;
+        T *q = out + s * L;
+        int64_t head = (int64_t)(((16 - ((uintptr_t)p & 15)) & 15) / sizeof(T));
+        if (head > L) head = L;
+        const int64_t nch = (L - head) / CH;          // whole chunks
+        const int64_t body_end = head + nch * CH;
+        // head: scalar, thread 0, in order
+        if (t == 0) {
+            V c = O::id();
+            for (int64_t j = 0; j < head; ++j) {
+                c = j == 0 ? O::lift(p[0], 0) : O::fold(c, p[j], j);
+                q[j] = O::val(c);
+                if (out_idx) out_idx[s * L + j] = O::idx(c);
+            }
+            s_carry = c;
+        }
+        __syncthreads();
+        V carry = s_carry;
+        int4 r[R], rn[R];
+        auto load = [&](int64_t ch, int4 (&dst)[R]) {
+            const int4 *src = reinterpret_cast<const int4 *>(p + head + ch * CH) + (int64_t)t * R;
+#pragma unroll
+            for (int k = 0; k < R; ++k) dst[k] = ldg16(src + k);
+        };
+        if (nch > 0) load(0, r);
+        for (int64_t ch = 0; ch < nch; ++ch) {
+            if (ch + 1 < nch) load(ch + 1, rn);
+            const int64_t j0 = head + ch * CH + (int64_t)t * E;  // row-local index of the thread's first element
+            V a[E];
+#pragma unroll
+            for (int k = 0; k < R; ++k) {
+                const Vec16<T> e = as_vec<T>(r[k]);
+#pragma unroll
+                for (int m = 0; m < VEC; ++m) {
+                    const int i = k * VEC + m;
+                    a[i] = i == 0 ? O::lift(e.e[0], j0) : O::fold(a[i - 1], e.e[m], j0 + i);
+                }
+            }
+            // block exclusive scan of the thread totals
+            V incl = a[E - 1];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const V y = shfl_up(incl, o);
+                if (lane >= o) incl = O::comb(y, incl);
+            }
+            V ex = shfl_up(incl, 1);
+            if (lane == 0) ex = O::id();
+            if (lane == 31) s_w[warp] = incl;
+            __syncthreads();
+            V wp = carry, tot = carry;
+#pragma unroll
+            for (int w = 0; w < 8; ++w) {
+                if (w < warp) wp = O::comb(wp, s_w[w]);
+                tot = O::comb(tot, s_w[w]);
+            }
+            __syncthreads();  // s_w is rewritten by the next chunk
+            const V pre = O::comb(wp, ex);
+            T *qo = q + head + ch * CH + (int64_t)t * E;
+#pragma unroll
+            for (int k = 0; k < R; ++k) {
+                Vec16<T> o;
+#pragma unroll
+                for (int m = 0; m < VEC; ++m) {
+                    const V z = O::comb(pre, a[k * VEC + m]);
+                    o.e[m] = O::val(z);
+                    if (out_idx) out_idx[s * L + j0 + k * VEC + m] = O::idx(z);
+                }
+                *reinterpret_cast<int4 *>(qo + k * VEC) = *reinterpret_cast<const int4 *>(&o);
+            }
+            carry = tot;
+#pragma unroll
+            for (int k = 0; k < R; ++k) r[k] = rn[k];
+        }
+        // ragged end: one partial chunk, element-guarded scalar loads, same block scan
+        if (body_end < L) {
+            const int64_t j0 = body_end + (int64_t)t * E;
+            V a[E];
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                const bool ok = j0 + i < L;
+                const V e = ok ? O::lift(p[j0 + i], j0 + i) : O::id();
+                a[i] = i == 0 ? e : O::comb(a[i - 1], e);
+            }
+            V incl = a[E - 1];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const V y = shfl_up(incl, o);
+                if (lane >= o) incl = O::comb(y, incl);
+            }
+            V ex = shfl_up(incl, 1);
+            if (lane == 0) ex = O::id();
+            if (lane == 31) s_w[warp] = incl;
+            __syncthreads();
+            V wp = carry;
+#pragma unroll
+            for (int w = 0; w < 8; ++w)
+                if (w < warp) wp = O::comb(wp, s_w[w]);
+            const V pre = O::comb(wp, ex);
+#pragma unroll
+            for (int i = 0; i < E; ++i)
+                if (j0 + i < L) {
+                    const V z = O::comb(pre, a[i]);
+                    q[j0 + i] = O::val(z);
+                    if (out_idx) out_idx[s * L + j0 + i] = O::idx(z);
+                }
+        }
+        __syncthreads();  // s_carry reuse
+    }
+}
+
+// KS2 applies when every SM gets several rows: the rows are then the unit of parallelism
+static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= 4 * (int64_t)sm_count(); }
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1117,6 +1247,18 @@ template <int OP, typename T> struct ScanRun {
                 const int64_t cap = resident_blocks((const void *)kb, 256);
                 grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
+                return launch_status();
+            }
+            constexpr int KS2R = (sizeof(T) == 4 && OP != kArgmin) ? 3 : 1;
+            constexpr int64_t KS2CH = 256 * KS2R * VEC;  // elements per chunk
+            // rows of >= 4 chunks (a row's partial last chunk is the slow, guarded part)
+            if (L >= 4 * KS2CH && nseg_ok(n, L) && !carry && map->ibase == 0 &&
+                ((((uintptr_t)in0) ^ ((uintptr_t)out)) & 15) == 0 && ((uintptr_t)in0 % sizeof(T)) == 0) {
+                auto kc = segscan_cta_kernel<OP, T, KS2R>;
+                const int64_t nseg = n / L;
+                int64_t grid = resident_blocks((const void *)kc, 256);
+                grid = grid > nseg ? nseg : grid;
+                kc<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, nseg, L, (T *)out, out_idx);
                 return launch_status();
             }
             if constexpr (OP != kArgmin) {  // (argmin's index output keeps the look-back path)

@@ -210,7 +210,8 @@ def test_workspace_queries_and_regimes(fs):
     assert r(64, 64, layout="col") == 4
     assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 5
     assert r(1 << 20, 3, scan=True) == 8 and r(1 << 20, 33, scan=True) == 5 and r(64, 7, scan=True, op="argmin") == 5
-    assert r(1 << 10, 2048, scan=True) == 5
+    assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 5  # KS2: >= 4 rows per SM
+    assert r(1 << 12, 2048, scan=True) == 5 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 9
     assert r(1 << 20, 512, scan=True, dtype=torch.int64) == 7 and r(1 << 20, 1024, scan=True, dtype=torch.int64) == 5
     assert r(0, 64) == 6 and r(64, 0) == 6
     assert r(64, 64, dtype=torch.int64, op="argmin") == 0

@@ -515,6 +515,24 @@ def test_seg_scan_short_rows_tile(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan tile {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("seglen", [2048, 4097, 12_289, 16_384, 65_537])
+def test_seg_scan_cta_rows(fs, seglen):
+    """KS2 (regime 9): a CTA owns whole rows (>= 4 rows per SM): whole and partial chunks,
+    misaligned row starts (odd lengths), argmin indices, int wrap-around; and a misaligned
+    view (head elements)."""
+    nseg = 4 * 148 + 7
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int64, "add"), (np.int32, "max")):
+        x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
+            workloads.mixed(nseg * seglen, nseg + seglen, dt)
+        if op == "argmin":
+            x[::9] = x.min()
+        got = fs.seg_scan(cu(x, 1 if seglen % 2 else 0), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan cta {nseg}x{seglen} {dt.__name__} {op}")
+
+
 def test_seg_scan_misaligned(fs):
     x = workloads.mixed(50 * 999, 4, np.int64)
     got = fs.seg_scan(cu(x, 1), 50, 999, "add")
