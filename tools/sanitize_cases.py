@@ -67,5 +67,9 @@ for nseg, L in ((1000, 8), (300, 33), (5, 20_000)):
     fs.seg_map_reduce(xi[: nseg * L], nseg, L, 2, "argmin")
 xb = cu(workloads.mixed(600 * 8192, 8, np.float32))  # CTA-per-row regime (>= 4 rows per SM)
 fs.seg_map_reduce(xb, 600, 8192, 1.0, "max")
+# seg_scan KS2 (CTA per row, running carry): whole + partial chunks, argmin, misaligned view
+xk = cu(workloads.mixed(600 * 12_289 + 1, 9, np.float32))
+fs.seg_scan(xk[: 600 * 12_289], 600, 12_289, "add")
+fs.seg_scan(xk[1:], 600, 12_289, "argmin")
 torch.cuda.synchronize()
 print("sanitize cases done")
