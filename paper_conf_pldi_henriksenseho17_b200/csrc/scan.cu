@@ -1167,8 +1167,10 @@ segscan_cta_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restri
     }
 }
 
-// KS2 applies when every SM gets several rows: the rows are then the unit of parallelism
-static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= 4 * (int64_t)sm_count(); }
+// KS2 applies when every SM gets at least one row: the rows are then the unit of parallelism
+// (seg sweep, profiles/r01_seg_sweep.json: at >= 1 row per SM KS2 beats the segmented look-back scan,
+// 256-268 rows 3.8 -> 4.8 TB/s, 512 rows 3.8 -> 4.5; below one row per SM SMs idle: 128 rows 3.6, 32 rows 1.1)
+static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm_count(); }
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,

@@ -488,6 +488,23 @@ def test_seg_scan_col_narrow(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan col narrow {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("nseg,seglen", [(128, 64), (128, 100_003), (256, 65), (1024, 1000), (4096, 3001),
+                                         (128 * 37, 777), (1 << 17, 64)])
+def test_seg_scan_col_wide(fs, nseg, seglen):
+    """Column-major seg_scan with wide rows (multiples of 128 four-byte columns, 16-byte
+    vectors): the three-pass kernels (partials, carries, scan) with ragged row blocks,
+    int wrap-around, 8-byte types and argmin."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int32, "min"), (np.float32, "max"),
+                   (np.float32, "min"), (np.int64, "add"), (np.float32, "argmin")):
+        x = workloads.mixed(nseg * seglen, nseg * 5 + seglen, dt)
+        if dt == np.int32 and op == "add":
+            x = workloads.full_range(x.size, seglen, np.int32)
+        got = fs.seg_scan(cu(x), nseg, seglen, op, layout="col")
+        want = oracle.seg_scan(x, nseg, seglen, op, "col")
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", "col") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan col wide {nseg}x{seglen} {dt.__name__} {op}")
+
+
 @pytest.mark.parametrize("seglen", [4, 64, 512])
 def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
     """KS0 needs 16-byte aligned buffers: a misaligned view takes the look-back scan and
