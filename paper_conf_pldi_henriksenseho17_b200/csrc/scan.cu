@@ -1171,6 +1171,10 @@ segscan_cta_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restri
 // (seg sweep, profiles/r01_seg_sweep.json: at >= 1 row per SM KS2 beats the segmented look-back scan,
 // 256-268 rows 3.8 -> 4.8 TB/s, 512 rows 3.8 -> 4.5; below one row per SM SMs idle: 128 rows 3.6, 32 rows 1.1)
 static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm_count(); }
+#ifndef FS_FLAT_ROW_MIN
+#define FS_FLAT_ROW_MIN (1 << 26)
+#endif
+constexpr int64_t kFlatRowMin = FS_FLAT_ROW_MIN;  // rows at least this long and fewer than the SMs: flat scan per row
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1276,6 +1280,18 @@ template <int OP, typename T> struct ScanRun {
                     kt<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, nseg, (int)L, (T *)out);
                     return launch_status();
                 }
+            }
+            // a few very long rows: each row is a flat scan (the unsegmented slab scan, one launch
+            // per row, workspace reused in stream order) -- fewer rows than SMs leave KS2 idle
+            // and the segmented look-back pays a head flag per tile
+            if (al && !carry && map->ibase == 0 && L >= kFlatRowMin && (L * (int64_t)sizeof(T)) % 16 == 0) {
+                for (int64_t s = 0; s < n / L; ++s) {
+                    const fs_status r = go<false, false, true>((const T *)in0 + s * L, nullptr, L, L, *map,
+                                                               (T *)out + s * L, out_idx ? out_idx + s * L : nullptr,
+                                                               nullptr, nullptr, ws, true, st);
+                    if (r != FS_OK) return r;
+                }
+                return FS_OK;
             }
             if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
             return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);

@@ -505,6 +505,21 @@ def test_seg_scan_col_wide(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan col wide {nseg}x{seglen} {dt.__name__} {op}")
 
 
+def test_seg_scan_few_long_rows(fs):
+    """Fewer rows than SMs, each >= 2^26 long and 16-byte aligned: one flat slab scan per
+    row (indices restart at every row: checked by argmin on the second row's ties)."""
+    nseg, seglen = 2, 1 << 26
+    for dt, op in ((np.float32, "add"), (np.int32, "max"), (np.int32, "argmin")):
+        x = workloads.mixed(nseg * seglen, 4242, dt)
+        if op == "argmin":
+            x[seglen + 5::9] = x.min()
+        got = fs.seg_scan(cu(x), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan long rows {nseg}x{seglen} {dt.__name__} {op}")
+        del got, want, asum
+
+
 @pytest.mark.parametrize("seglen", [4, 64, 512])
 def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
     """KS0 needs 16-byte aligned buffers: a misaligned view takes the look-back scan and
