@@ -931,13 +931,18 @@ segscan_vec_kernel(const T *__restrict__ x, int64_t n, int L, int G, T *__restri
 // segments); every lane scans its vector in registers, every warp scans its lane totals
 // with shuffles, and the warps of a segment combine their totals through shared memory
 // (one barrier per U chunks).  No look-back, no flags: one read, one write per element.
-template <int OP, typename T, int U>
+// BIG: rows of 2..U chunks (256 * VEC < L <= U * 256 * VEC, U = 4 or 8); a row's warps then
+// span chunks of one step, and warp 0 scans the U * 8 warp totals (segmented by row, U / 4
+// totals per lane).
+template <int OP, typename T, int U, bool BIG = false>
 __global__ void __launch_bounds__(256)
 segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ out, int64_t *__restrict__ out_idx) {
     using O = Op<OP, T>;
     using V = typename O::V;
     constexpr int VEC = 16 / sizeof(T);
+    static_assert(!BIG || U == 4 || U == 8, "one warp scans the step's U * 8 warp totals, 1 or 2 per lane");
     __shared__ V wt[U][8];
+    __shared__ V wx[BIG ? U * 8 : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int WS = L / (32 * VEC);          // warps per segment (2, 4 or 8)
     const int wr = warp & (WS - 1);         // rank of this warp within its segment
@@ -952,7 +957,8 @@ segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ ou
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const Vec16<T> e = as_vec<T>(r[u]);
-            const int j0 = (wr * 32 + lane) * VEC;  // segment-local index of the first element
+            const int wru = BIG ? ((u * 8 + warp) & (WS - 1)) : wr;
+            const int j0 = (wru * 32 + lane) * VEC;  // segment-local index of the first element
 #pragma unroll
             for (int k = 0; k < VEC; ++k)
                 a[u][k] = k == 0 ? O::lift(e.e[0], j0) : O::fold(a[u][k - 1], e.e[k], j0 + k);
@@ -967,13 +973,35 @@ segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ ou
             if (lane == 31) wt[u][warp] = incl;
         }
         __syncthreads();
+        if constexpr (BIG) {
+            if (warp == 0) {
+                constexpr int P = U / 4;           // warp totals per lane (a pair never straddles a row: WS >= 16)
+                const int rk = lane & (WS / P - 1);  // rank of this lane's totals within their row
+                const V t0 = (&wt[0][0])[lane * P];
+                const V t1 = P == 2 ? (&wt[0][0])[lane * P + P - 1] : O::id();
+                V incl = P == 2 ? O::comb(t0, t1) : t0;
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            V p = O::id();
-            for (int q = warp - wr; q < warp; ++q) p = O::comb(p, wt[u][q]);
-            ex[u] = O::comb(p, ex[u]);
+                for (int dd = 1; dd < 32; dd <<= 1) {
+                    const V y = shfl_up(incl, dd);
+                    if (rk >= dd) incl = O::comb(y, incl);
+                }
+                V e = shfl_up(incl, 1);
+                if (rk == 0) e = O::id();
+                wx[lane * P] = e;
+                if (P == 2) wx[lane * P + 1] = O::comb(e, t0);
+            }
+            __syncthreads();
+#pragma unroll
+            for (int u = 0; u < U; ++u) ex[u] = O::comb(wx[u * 8 + warp], ex[u]);
+        } else {
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                V p = O::id();
+                for (int q = warp - wr; q < warp; ++q) p = O::comb(p, wt[u][q]);
+                ex[u] = O::comb(p, ex[u]);
+            }
         }
-        __syncthreads();  // wt is reused by the next chunks
+        __syncthreads();  // wt / wx are reused by the next chunks
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const int64_t v = (c0 + u) * 256 + threadIdx.x;
@@ -1250,6 +1278,16 @@ template <int OP, typename T> struct ScanRun {
                 auto kb = segscan_blk_kernel<OP, T, 2>;
                 const int64_t nchunk = ceil_div(n / VEC, 256);
                 int64_t grid = ceil_div(nchunk > 0 ? nchunk : 1, 2);
+                const int64_t cap = resident_blocks((const void *)kb, 256);
+                grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
+                kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
+                return launch_status();
+            }
+            if (al && !carry && map->ibase == 0 && L > 256 * VEC && L <= 2048 * VEC && (L & (L - 1)) == 0) {
+                const bool u8 = L > 1024 * VEC;
+                auto kb = u8 ? segscan_blk_kernel<OP, T, 8, true> : segscan_blk_kernel<OP, T, 4, true>;
+                const int64_t nchunk = ceil_div(n / VEC, 256);
+                int64_t grid = ceil_div(nchunk > 0 ? nchunk : 1, u8 ? 8 : 4);
                 const int64_t cap = resident_blocks((const void *)kb, 256);
                 grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);

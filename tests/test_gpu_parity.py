@@ -450,12 +450,13 @@ def test_seg_scan(fs, nseg, seglen, layout):
         assert_reduced(got, want, op, asum, f"segscan {layout} {nseg}x{seglen} {dt.__name__} {op}")
 
 
-@pytest.mark.parametrize("seglen", [1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024])
+@pytest.mark.parametrize("seglen", [1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192])
 @pytest.mark.parametrize("nseg", [1, 3, 1001, 7_001])
 def test_seg_scan_short_pow2(fs, nseg, seglen):
     """KS0 (regime 7): power-of-two rows by in-register + shuffle scans (one warp) and a
-    shared-memory combine across warps (256..1024 f32, 128..512 8-byte); every op and
-    dtype (8-byte types at 1024 go to the look-back scan), ragged vector tails for
+    shared-memory combine across warps (256..1024 f32, 128..512 8-byte), rows of 2-8
+    chunks (2048..8192 f32, 1024..4096 8-byte; 8-byte 8192 takes the look-back scan); every
+    op and dtype, ragged vector tails for
     L < 4, argmin ties, int wrap-around."""
     for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
                    (np.int32, "max"), (np.int64, "add"), (np.int64, "argmin"), (np.float32, "max")):
