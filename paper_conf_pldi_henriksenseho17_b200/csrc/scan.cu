@@ -1018,6 +1018,91 @@ segscan_blk_kernel(const T *__restrict__ x, int64_t n, int L, T *__restrict__ ou
     }
 }
 
+// KS3: rows of any length 32 < L <= 16384 (non-powers of two, whose 16-byte vectors straddle
+// rows): a CTA takes R whole rows (R * L ~ 8192 elements) at a time, so no scan crosses a CTA
+// and there is no look-back.  The rows are staged in shared memory by coalesced loads, each
+// thread scans a contiguous piece sequentially (restarting at row heads), the CTA scans the
+// 256 (head seen, total) piece summaries, each piece's first partial row takes its carry, and
+// the rows leave by coalesced stores.  ADD/MIN/MAX (argmin's index output keeps the look-back).
+constexpr int kRowsElems = 8192;
+template <int OP, typename T>
+__global__ void __launch_bounds__(256)
+segscan_rows_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, int64_t R, T *__restrict__ out) {
+    using O = Op<OP, T>;
+    extern __shared__ __align__(16) unsigned char smem_rows[];
+    T *buf = reinterpret_cast<T *>(smem_rows);
+    __shared__ T s_wa[8];
+    __shared__ int s_wf[8];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t nchunk = (nseg + R - 1) / R;
+    for (int64_t c = blockIdx.x; c < nchunk; c += gridDim.x) {
+        const int64_t r0 = c * R, rows = (r0 + R < nseg ? r0 + R : nseg) - r0;
+        const int cnt = (int)(rows * L);
+        const T *src = x + r0 * L;
+#pragma unroll 8
+        for (int i = tid; i < cnt; i += 256) buf[i] = __ldcs(src + i);
+        __syncthreads();
+        const int E = ((cnt + 255) / 256) | 1;  // odd piece length: the lanes' strided reads hit distinct banks
+        const int i0 = tid * E < cnt ? tid * E : cnt, i1 = i0 + E < cnt ? i0 + E : cnt;
+        int j = (int)(i0 % L);  // position of element i0 in its row
+        T acc = O::id();
+        int f = 0;  // a row head lies in this piece
+        for (int i = i0; i < i1; ++i) {
+            const T v = buf[i];
+            if (j == 0) {
+                acc = v;
+                f = 1;
+            } else {
+                acc = O::comb(acc, v);
+            }
+            buf[i] = acc;
+            if (++j == L) j = 0;
+        }
+        // inclusive segmented scan of the (f, acc) piece summaries: (f1,a1).(f2,a2) = (f1|f2, f2 ? a2 : a1.a2)
+        T a = acc;
+        int fl = f;
+#pragma unroll
+        for (int dd = 1; dd < 32; dd <<= 1) {
+            const T ya = shfl_up(a, dd);
+            const int yf = __shfl_up_sync(0xffffffffu, fl, dd);
+            if (lane >= dd) {
+                if (!fl) a = O::comb(ya, a);
+                fl |= yf;
+            }
+        }
+        if (lane == 31) {
+            s_wa[warp] = a;
+            s_wf[warp] = fl;
+        }
+        __syncthreads();
+        // exclusive prefix of this piece = (warps before, combined in order) . (lanes before in this warp)
+        T ex = shfl_up(a, 1);
+        int exf = __shfl_up_sync(0xffffffffu, fl, 1);
+        if (lane == 0) {
+            ex = O::id();
+            exf = 0;
+        }
+        if (!exf) {
+            T p = O::id();
+            for (int q = 0; q < warp; ++q) p = s_wf[q] ? s_wa[q] : O::comb(p, s_wa[q]);
+            ex = O::comb(p, ex);
+        }
+        // the piece's elements before its first row head continue the previous piece's row
+        {
+            int jj = (int)(i0 % L);
+            for (int i = i0; i < i1 && jj != 0; ++i) {
+                buf[i] = O::comb(ex, buf[i]);
+                if (++jj == L) jj = 0;
+            }
+        }
+        __syncthreads();
+        T *dst = out + r0 * L;
+#pragma unroll 8
+        for (int i = tid; i < cnt; i += 256) __stcs(dst + i, buf[i]);
+        __syncthreads();  // buf / s_wa reused by the next chunk
+    }
+}
+
 // KS1: short rows of any length L <= 32 that are not powers of two (a 16-byte vector then
 // straddles rows): a CTA stages 256 whole rows through shared memory with coalesced 16-byte
 // loads (index padded every 32 elements), thread t scans row t sequentially in place, and
@@ -1306,6 +1391,20 @@ template <int OP, typename T> struct ScanRun {
                 return launch_status();
             }
             if constexpr (OP != kArgmin) {  // (argmin's index output keeps the look-back path)
+                if (!carry && map->ibase == 0 && L > 32 && L <= (sizeof(T) == 4 ? 16384 : 8192) &&
+                    ((uintptr_t)in0 % sizeof(T)) == 0 && ((uintptr_t)out % sizeof(T)) == 0) {
+                    auto kr = segscan_rows_kernel<OP, T>;
+                    const int64_t nseg = n / L;
+                    const int64_t R = L >= kRowsElems ? 1 : kRowsElems / L;
+                    const int smem = (int)(R * L * (int64_t)sizeof(T));
+                    if (smem > 48 * 1024)
+                        cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                    int64_t grid = ceil_div(nseg, R);
+                    const int64_t cap = resident_blocks((const void *)kr, 256, (size_t)smem);
+                    grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
+                    kr<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, nseg, L, R, (T *)out);
+                    return launch_status();
+                }
                 if (al && !carry && map->ibase == 0 && L >= 2 && L <= 32) {
                     auto kt = segscan_tile_kernel<OP, T>;
                     const int smem = (int)((256 * L + 256 * L / 32 + 1) * sizeof(T));

@@ -548,6 +548,23 @@ def test_seg_scan_short_rows_tile(fs, nseg, seglen):
         assert_reduced(got, want, op, asum, f"segscan tile {nseg}x{seglen} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("seglen", [33, 100, 1000, 1023, 4097, 8191, 9000, 16_383])
+@pytest.mark.parametrize("nseg,offset", [(1, 0), (7, 1), (1001, 0), (300, 3)])
+def test_seg_scan_rows_ks3(fs, nseg, seglen, offset):
+    """KS3: rows of 32 < L <= 16384 (8192 for 8-byte types) staged R whole rows per CTA in
+    shared memory: several rows per CTA and a row per CTA, pieces that straddle row heads,
+    a partial last chunk, misaligned views, int wrap-around; argmin and long 8-byte rows
+    keep the look-back scan."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int64, "add"),
+                   (np.int32, "max"), (np.float32, "min"), (np.float32, "argmin")):
+        x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
+            workloads.mixed(nseg * seglen, nseg * 13 + seglen, dt)
+        got = fs.seg_scan(cu(x, offset), nseg, seglen, op)
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan ks3 {nseg}x{seglen}+{offset} {dt.__name__} {op}")
+
+
 @pytest.mark.parametrize("seglen", [2048, 4097, 12_289, 16_384, 65_537])
 def test_seg_scan_cta_rows(fs, seglen):
     """KS2 (regime 9): a CTA owns whole rows (>= 4 rows per SM): whole and partial chunks,
