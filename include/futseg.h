@@ -275,32 +275,52 @@ fs_status fs_scan_reduce(int32_t scan_op, int32_t red_op, int32_t dtype, const v
  * Returns FS_ERR_BOUNDS if a kernel flagged a precondition violation. */
 fs_status fs_check_device_error(void *ws, void *stream);
 
-/* Regime the dispatcher picks for a segmented call on the current device:
- *   0 = KG1 thread-per-segment over a shared-memory tile (short rows)
- *   1 = KG2 warp per segment
- *   2 = KG3 block per segment
- *   3 = KG4 several blocks per segment, partials combined by the last block
- *   4 = column kernel (FS_COL_MAJOR: thread per segment, coalesced rows)
- *   5 = single-pass segmented look-back scan (fs_seg_scan, FS_ROW_MAJOR)
- *   6 = empty input (neutral fill)
- *   7 = KS0 fs_seg_scan of power-of-two rows up to 256 16-byte vectors (seglen <=
- *       256 * 16/sizeof(elem), FS_ROW_MAJOR, 16-byte aligned buffers; others take 5):
- *       in-register scan, shuffle scan across the lanes of a segment and, for rows
- *       longer than a warp's 32 vectors, a shared-memory combine across its warps
- *   8 = KS1 fs_seg_scan of short rows that are not powers of two (seglen <= 32,
- *       FS_ROW_MAJOR, 16-byte aligned, op != ARGMIN): 256 rows staged through shared
- *       memory, a thread scans a row
- *   9 = KS2 fs_seg_scan of long rows (at least 4 chunks of 256 x R vectors: 12288 f32,
- *       4096 f32 argmin, 2048 8-byte elements) when there are at least
- *       4 rows per SM (FS_ROW_MAJOR, in/out with the same 16-byte phase): a CTA owns
- *       whole rows and scans them chunk by chunk with a running carry (no look-back)
+/* Run-time multi-versioning (the paper's future work, L1411-1418): the segmented
+ * primitives pick a kernel by segment length.  Regime IDs (FS_REGIME_*):
+ *   0 = KG0/KG1 short rows: power-of-two rows by in-lane + shuffle groups over
+ *       16-byte loads (KG0), others thread/group per segment over a shared-memory
+ *       tile (KG1)                                                     fs_seg_reduce
+ *   1 = KG2 warp per segment                                            fs_seg_reduce
+ *   2 = KG3 block per segment                                           fs_seg_reduce
+ *   3 = KG4 several blocks per segment, partials combined by the last   fs_seg_reduce
+ *   4 = column kernels (FS_COL_MAJOR with nseg > 1 and seglen > 1)      both
+ *   5 = single-pass segmented decoupled-look-back slab scan (the general
+ *       case: argmin, carries, misaligned buffers, lengths no other regime takes)
+ *   6 = empty input (nseg == 0 or seglen == 0: neutral fill / nothing)  both
+ *   7 = KS0 power-of-two rows of <= 256 16-byte vectors (seglen <= 1024 f32/i32,
+ *       512 i64), 16-byte aligned buffers: in-register + shuffle scan, a shared-memory
+ *       combine across the warps of a CTA for rows longer than 32 vectors
+ *   8 = KS1 rows of 2..32 elements that are not powers of two, op != ARGMIN, 16-byte
+ *       aligned: 256 rows staged through shared memory, a thread scans a row
+ *   9 = KS2 rows of >= 4 chunks of 256 x R vectors (12288 f32/i32 add/min/max, 4096
+ *       argmin, 2048 i64) when there are at least as many rows as SMs (in/out with the
+ *       same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with a
+ *       running carry (no look-back)
+ *  10 = KS0-BIG power-of-two rows of 2-8 CTA steps (256 < seglen/VEC <= 2048: 2048..8192
+ *       f32/i32, 1024..4096 i64), 16-byte aligned: a CTA loads a whole row per step,
+ *       warp 0 scans the warp totals
+ *  11 = KS3 rows of 32 < seglen <= 16384 (8192 for i64), op != ARGMIN, element-aligned:
+ *       R whole rows per CTA staged in shared memory, odd-length per-thread pieces, a
+ *       CTA scan of the piece summaries (no look-back)
+ *  12 = flat (unsegmented) slab scan per row: one row (nseg == 1), or fewer rows than SMs
+ *       of >= 2^26 elements each, 16-byte aligned
+ * fs_seg_regime returns the regime a call with these sizes takes on the current device
+ * when its buffers come from an allocator (16-byte aligned); misaligned views may take
+ * 5 instead.  The row-major seg_scan plan is one function shared with the dispatcher.
  * Returns -1 for invalid arguments. */
 int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen,
                       int32_t layout);
 
-/* Testing / sweep aid: force the seg_reduce regime (0..3 for FS_ROW_MAJOR) for
- * subsequent calls in this process; -1 restores automatic selection.  Also
- * settable with the environment variable FUTSEG_FORCE_REGIME. */
+/* The regime the last fs_seg_reduce / fs_seg_scan call made BY THIS HOST THREAD actually
+ * launched (-1 before any call).  Test aid: asserts that fs_seg_regime tells the truth. */
+int32_t fs_last_seg_regime(void);
+
+/* Testing / sweep aid: force a regime for subsequent calls in this process; -1
+ * restores automatic selection.  0..3 force the FS_ROW_MAJOR seg_reduce regime;
+ * 5 and 7..12 force a row-major seg_scan regime wherever its preconditions above hold
+ * (elsewhere the automatic choice stands; forced 12 drops its 2^26 length threshold).
+ * Also settable with the environment variable FUTSEG_FORCE_REGIME.  Returns
+ * FS_ERR_UNSUPPORTED for other values. */
 fs_status fs_force_seg_regime(int32_t regime);
 
 const char *fs_status_string(fs_status s);

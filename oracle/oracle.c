@@ -27,8 +27,11 @@
  *   R5 NN distance map: sqrtf((lat-q0)*(lat-q0) + (lng-q1)*(lng-q1)) with
  *      every operation separately rounded to f32 (built -ffp-contract=off).
  *
- * Build: gcc -O2 -ffp-contract=off -fno-fast-math -shared -fPIC (see
- * oracle/build.sh).  Status codes: 0 ok, 1 bad argument, 2 key out of range.
+ * Build: gcc -O2 -ffp-contract=off -fno-fast-math -std=c11 -shared -fPIC (the
+ * command is oracle/__init__.py build()).  -ffp-contract=off makes every a*b+c
+ * below two roundings; the one fused multiply-add the oracle wants (R18,
+ * orc_kmeans_step) is an explicit fmaf().  Status codes: 0 ok, 1 bad argument,
+ * 2 key out of range.
  */
 #include <math.h>
 #include <stdint.h>

@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "last_seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -42,10 +42,11 @@ OPS = {"add": 0, "min": 1, "max": 2, "argmin": 3, "vadd": 4}
 MAPS = {"id": 0, "nn_dist": 1}
 LAYOUTS = {"row": 0, "col": 1}
 _DT = {torch.int32: FS_I32, torch.int64: FS_I64, torch.float32: FS_F32}
-REGIMES = {0: "KG1 smem tile", 1: "KG2 warp/segment", 2: "KG3 block/segment", 3: "KG4 multi-block/segment",
-           4: "column (col-major)", 5: "segmented look-back scan", 6: "empty",
+REGIMES = {0: "KG0/KG1 short rows (shuffle groups / smem tile)", 1: "KG2 warp/segment", 2: "KG3 block/segment",
+           3: "KG4 multi-block/segment", 4: "column (col-major)", 5: "segmented look-back scan", 6: "empty",
            7: "KS0 short power-of-two scan (register + shuffle)", 8: "KS1 short-row scan (shared-memory tile)",
-           9: "KS2 CTA-per-row scan with a running carry"}
+           9: "KS2 CTA-per-row scan with a running carry", 10: "KS0-BIG power-of-two rows of 2-8 CTA steps",
+           11: "KS3 whole rows staged in shared memory", 12: "flat slab scan per row"}
 
 
 class fs_opdesc(ctypes.Structure):
@@ -82,6 +83,7 @@ _SIG = {
     "fs_check_device_error": [_P, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
+    "fs_last_seg_regime": [],
     "fs_status_string": [_I],
     "fs_version": [],
     "fs_launch_count": [],
@@ -414,6 +416,11 @@ def check_device_error(device=None):
 def seg_regime(nseg: int, seglen: int, op: str = "add", dtype=torch.float32, layout: str = "row",
                scan: bool = False) -> int:
     return int(_lib.fs_seg_regime(1 if scan else 0, _op(op, _DT[dtype]), nseg, seglen, LAYOUTS[layout]))
+
+
+def last_seg_regime() -> int:
+    """The regime the last seg_reduce / seg_scan call of this thread launched (include/futseg.h)."""
+    return int(_lib.fs_last_seg_regime())
 
 
 def force_seg_regime(regime: int):

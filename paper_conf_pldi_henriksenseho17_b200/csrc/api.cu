@@ -57,6 +57,10 @@ int forced_seg_regime() {
     return g_forced_regime;
 }
 
+static thread_local int g_last_regime = -1;
+void note_regime(int r) { g_last_regime = r; }
+int last_regime() { return g_last_regime; }
+
 }  // namespace fs
 
 using namespace fs;
@@ -150,7 +154,9 @@ const char *fs_status_string(fs_status s) {
 }
 
 fs_status fs_force_seg_regime(int32_t regime) {
-    if (regime < -1 || regime > 3) return FS_ERR_UNSUPPORTED;
+    // -1 automatic; 0..3 the seg_reduce regimes; 5, 7..12 the row-major seg_scan regimes
+    // (applied only where their preconditions hold, see fs::seg_scan_plan)
+    if (regime < -1 || regime == 4 || regime == 6 || regime > 12) return FS_ERR_UNSUPPORTED;
     g_forced_regime = regime;
     return FS_OK;
 }
@@ -326,9 +332,11 @@ fs_status fs_seg_reduce(fs_opdesc op, const void *in, int64_t nseg, int64_t segl
     FS_TRY(fs_seg_reduce_workspace(op, nseg, seglen, layout, &need));
     FS_TRY(check_ws(ws, ws_bytes, need));
     int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
+    note_regime(RG_EMPTY);
     if (nseg == 0) return FS_OK;
     if (seglen == 0) return fill_neutral_run(op.op, op.dtype, nseg, out, oi, S(stream));
     // with one segment, or segments of one element, both layouts are the same bytes
+    note_regime(RG_COL);
     if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1)
         return colreduce_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
     return seg_reduce_run(op.op, op.dtype, in, nseg, seglen, out, oi, ws, S(stream));
@@ -341,7 +349,9 @@ fs_status fs_seg_scan(fs_opdesc op, const void *in, int64_t nseg, int64_t seglen
     FS_TRY(fs_seg_scan_workspace(op, nseg, seglen, layout, &need));
     FS_TRY(check_ws(ws, ws_bytes, need));
     int64_t *oi = op.op == FS_ARGMIN ? out_idx : nullptr;
+    note_regime(RG_EMPTY);
     if (nseg * seglen == 0) return FS_OK;
+    note_regime(RG_COL);
     if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1)
         return colscan_run(op.op, op.dtype, in, seglen, nseg, out, oi, ws, S(stream));
     const fs_mapdesc id = {FS_MAP_ID, 0.f, 0.f, 0};
@@ -506,17 +516,13 @@ fs_status fs_check_device_error(void *ws, void *stream) {
 int32_t fs_seg_regime(int32_t prim_is_scan, fs_opdesc op, int64_t nseg, int64_t seglen, int32_t layout) {
     if (check_op(op, false) != FS_OK || nseg < 0 || seglen < 0 || mul_overflows(nseg, seglen)) return -1;
     if (layout != FS_ROW_MAJOR && layout != FS_COL_MAJOR) return -1;
-    if (nseg == 0 || seglen == 0) return 6;
-    if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1) return 4;
-    if (prim_is_scan) {
-        const int64_t vec = 16 / (int64_t)dtype_size(op.dtype);
-        if (nseg > 1 && (seglen & (seglen - 1)) == 0 && seglen <= 256 * vec) return 7;
-        if (nseg > 1 && seglen >= 2 && seglen <= 32 && op.op != FS_ARGMIN) return 8;
-        const int64_t ks2ch = 256 * vec * ((dtype_size(op.dtype) == 4 && op.op != FS_ARGMIN) ? 3 : 1);
-        if (seglen >= 4 * ks2ch && nseg >= 4 * (int64_t)sm_count()) return 9;
-        return 5;
-    }
+    if (nseg == 0 || seglen == 0) return RG_EMPTY;
+    if (layout == FS_COL_MAJOR && nseg > 1 && seglen > 1) return RG_COL;
+    if (prim_is_scan)  // buffers from an allocator: 16-byte aligned, same phase
+        return seg_scan_plan(op.op, op.dtype, nseg * seglen, seglen, true, true, true, true);
     return seg_reduce_regime(op.op, op.dtype, nseg, seglen);
 }
+
+int32_t fs_last_seg_regime(void) { return fs::last_regime(); }
 
 }  // extern "C"

@@ -17,6 +17,19 @@ inline int resident_blocks(const void *kernel, int threads, size_t smem = 0) {
     return sm_count() * max_blocks_per_sm(kernel, threads, smem);
 }
 int forced_seg_regime();  // -1 = automatic
+void note_regime(int r);   // the segmented regime the current call launched (fs_last_seg_regime)
+
+// Segmented-regime IDs (include/futseg.h FS_REGIME_*): the one numbering shared by the
+// dispatchers, fs_seg_regime and fs_last_seg_regime.
+enum {
+    RG_KG1 = 0, RG_KG2 = 1, RG_KG3 = 2, RG_KG4 = 3, RG_COL = 4, RG_KS_LOOKBACK = 5, RG_EMPTY = 6,
+    RG_KS0 = 7, RG_KS1 = 8, RG_KS2 = 9, RG_KS0_BIG = 10, RG_KS3 = 11, RG_FLAT_ROW = 12
+};
+// Row-major seg_scan regime for n = nseg * L elements (nseg >= 1, L >= 1): the single plan both
+// ScanRun (scan.cu) and fs_seg_regime use.  al16: in and out 16-byte aligned; co16: in and out
+// share their 16-byte phase; elem: in and out aligned to the element size; plain: no carry-in
+// and ibase 0 (every seg_scan call).
+int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bool elem, bool plain);
 
 void note_launches(int n);  // counts kernels launched by this library (fs_launch_count)
 inline fs_status launch_status(int kernels = 1) {

@@ -25,6 +25,8 @@
 // blocks are chained by a reduce / exclusive-scan-of-partials / rescan.
 #include <stdlib.h>
 
+#include <type_traits>
+
 #include "internal.cuh"
 
 namespace fs {
@@ -1288,6 +1290,44 @@ static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm
 #define FS_FLAT_ROW_MIN (1 << 26)
 #endif
 constexpr int64_t kFlatRowMin = FS_FLAT_ROW_MIN;  // rows at least this long and fewer than the SMs: flat scan per row
+template <int OP, typename T> constexpr int ks2_rows() { return (sizeof(T) == 4 && OP != kArgmin) ? 3 : 1; }
+template <typename T> constexpr int dt_of() {
+    return sizeof(T) == 8 ? FS_I64 : (std::is_same<T, float>::value ? FS_F32 : FS_I32);
+}
+
+// The row-major seg_scan plan (internal.cuh).  Natural order: KS0 (power-of-two rows that fit one
+// CTA step), KS0-BIG (power-of-two rows of 2-8 steps), KS2 (rows of >= 4 chunks, >= 1 row per SM),
+// KS3 (32 < L <= 16384 staged in shared memory), KS1 (L <= 32 staged), the flat slab scan per
+// row (rows >= kFlatRowMin, fewer than the SMs), else the segmented look-back scan.  A regime
+// forced with fs_force_seg_regime is taken when its preconditions hold (the flat per-row scan
+// then drops its length threshold).
+int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bool elem, bool plain) {
+    if (L >= n) return RG_FLAT_ROW;  // one row: the unsegmented scan
+    const int64_t es = (int64_t)dtype_size(dt), VEC = 16 / es;
+    const bool pow2 = (L & (L - 1)) == 0;
+    const int64_t ks2ch = 256 * VEC * ((es == 4 && op != FS_ARGMIN) ? 3 : 1);
+    const bool ok[13] = {
+        false, false, false, false, false,
+        true,                                                                         // 5 look-back
+        false,
+        al16 && plain && pow2 && L <= 256 * VEC,                                      // 7 KS0
+        op != FS_ARGMIN && al16 && plain && L >= 2 && L <= 32,                        // 8 KS1
+        plain && co16 && elem && L >= 4 * ks2ch && nseg_ok(n, L),                     // 9 KS2
+        al16 && plain && pow2 && L > 256 * VEC && L <= 2048 * VEC,                    // 10 KS0-BIG
+        op != FS_ARGMIN && plain && elem && L > 32 && L <= (es == 4 ? 16384 : 8192),  // 11 KS3
+        al16 && plain && (L * es) % 16 == 0,                                          // 12 flat per row
+    };
+    const int f = forced_seg_regime();
+    if (f >= 5 && f <= 12 && ok[f]) return f;
+    if (ok[RG_KS0]) return RG_KS0;
+    if (ok[RG_KS0_BIG]) return RG_KS0_BIG;
+    if (ok[RG_KS2]) return RG_KS2;
+    if (ok[RG_KS3]) return RG_KS3;
+    if (ok[RG_KS1]) return RG_KS1;
+    if (ok[RG_FLAT_ROW] && L >= kFlatRowMin) return RG_FLAT_ROW;
+    return RG_KS_LOOKBACK;
+}
+
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1349,7 +1389,12 @@ template <int OP, typename T> struct ScanRun {
         }
         if (seg) {
             constexpr int64_t VEC = 16 / sizeof(T);
-            if (al && !carry && map->ibase == 0 && L >= 1 && L <= 32 * VEC && (L & (L - 1)) == 0) {
+            const bool co16 = ((((uintptr_t)in0) ^ ((uintptr_t)out)) & 15) == 0;
+            const bool elem = ((uintptr_t)in0 % sizeof(T)) == 0 && ((uintptr_t)out % sizeof(T)) == 0;
+            const bool plain = !carry && map->ibase == 0;
+            const int rg = seg_scan_plan(OP, dt_of<T>(), n, L, al, co16, elem, plain);
+            note_regime(rg);
+            if (rg == RG_KS0 && L <= 32 * VEC) {
                 auto kv = segscan_vec_kernel<OP, T, 4>;
                 const int64_t nvec = n / VEC;
                 int64_t grid = ceil_div(nvec > 0 ? nvec : 1, 256 * 4);
@@ -1359,7 +1404,7 @@ template <int OP, typename T> struct ScanRun {
                 kv<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, G, (T *)out, out_idx);
                 return launch_status();
             }
-            if (al && !carry && map->ibase == 0 && L > 32 * VEC && L <= 256 * VEC && (L & (L - 1)) == 0) {
+            if (rg == RG_KS0) {
                 auto kb = segscan_blk_kernel<OP, T, 2>;
                 const int64_t nchunk = ceil_div(n / VEC, 256);
                 int64_t grid = ceil_div(nchunk > 0 ? nchunk : 1, 2);
@@ -1368,7 +1413,7 @@ template <int OP, typename T> struct ScanRun {
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
                 return launch_status();
             }
-            if (al && !carry && map->ibase == 0 && L > 256 * VEC && L <= 2048 * VEC && (L & (L - 1)) == 0) {
+            if (rg == RG_KS0_BIG) {
                 const bool u8 = L > 1024 * VEC;
                 auto kb = u8 ? segscan_blk_kernel<OP, T, 8, true> : segscan_blk_kernel<OP, T, 4, true>;
                 const int64_t nchunk = ceil_div(n / VEC, 256);
@@ -1378,11 +1423,8 @@ template <int OP, typename T> struct ScanRun {
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
                 return launch_status();
             }
-            constexpr int KS2R = (sizeof(T) == 4 && OP != kArgmin) ? 3 : 1;
-            constexpr int64_t KS2CH = 256 * KS2R * VEC;  // elements per chunk
-            // rows of >= 4 chunks (a row's partial last chunk is the slow, guarded part)
-            if (L >= 4 * KS2CH && nseg_ok(n, L) && !carry && map->ibase == 0 &&
-                ((((uintptr_t)in0) ^ ((uintptr_t)out)) & 15) == 0 && ((uintptr_t)in0 % sizeof(T)) == 0) {
+            if (rg == RG_KS2) {
+                constexpr int KS2R = ks2_rows<OP, T>();
                 auto kc = segscan_cta_kernel<OP, T, KS2R>;
                 const int64_t nseg = n / L;
                 int64_t grid = resident_blocks((const void *)kc, 256);
@@ -1391,8 +1433,7 @@ template <int OP, typename T> struct ScanRun {
                 return launch_status();
             }
             if constexpr (OP != kArgmin) {  // (argmin's index output keeps the look-back path)
-                if (!carry && map->ibase == 0 && L > 32 && L <= (sizeof(T) == 4 ? 16384 : 8192) &&
-                    ((uintptr_t)in0 % sizeof(T)) == 0 && ((uintptr_t)out % sizeof(T)) == 0) {
+                if (rg == RG_KS3) {
                     auto kr = segscan_rows_kernel<OP, T>;
                     const int64_t nseg = n / L;
                     const int64_t R = L >= kRowsElems ? 1 : kRowsElems / L;
@@ -1405,7 +1446,7 @@ template <int OP, typename T> struct ScanRun {
                     kr<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, nseg, L, R, (T *)out);
                     return launch_status();
                 }
-                if (al && !carry && map->ibase == 0 && L >= 2 && L <= 32) {
+                if (rg == RG_KS1) {
                     auto kt = segscan_tile_kernel<OP, T>;
                     const int smem = (int)((256 * L + 256 * L / 32 + 1) * sizeof(T));
                     if (smem > 48 * 1024)
@@ -1421,7 +1462,7 @@ template <int OP, typename T> struct ScanRun {
             // a few very long rows: each row is a flat scan (the unsegmented slab scan, one launch
             // per row, workspace reused in stream order) -- fewer rows than SMs leave KS2 idle
             // and the segmented look-back pays a head flag per tile
-            if (al && !carry && map->ibase == 0 && L >= kFlatRowMin && (L * (int64_t)sizeof(T)) % 16 == 0) {
+            if (rg == RG_FLAT_ROW) {
                 for (int64_t s = 0; s < n / L; ++s) {
                     const fs_status r = go<false, false, true>((const T *)in0 + s * L, nullptr, L, L, *map,
                                                                (T *)out + s * L, out_idx ? out_idx + s * L : nullptr,
@@ -1433,6 +1474,7 @@ template <int OP, typename T> struct ScanRun {
             if (al) return go<false, true, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
             return go<false, true, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
         }
+        note_regime(RG_FLAT_ROW);
         if (al) return go<false, false, true>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
         return go<false, false, false>(in0, in1, n, L, *map, out, out_idx, carry, carry_idx, ws, al, st);
     }

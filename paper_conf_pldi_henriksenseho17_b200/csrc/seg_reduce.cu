@@ -499,6 +499,7 @@ size_t seg_reduce_ws(int op, int dt, int64_t nseg, int64_t L) {
 fs_status seg_reduce_run(int op, int dt, const void *in, int64_t nseg, int64_t L, void *out, int64_t *out_idx,
                          void *ws, cudaStream_t st) {
     const int regime = seg_reduce_regime(op, dt, nseg, L);
+    note_regime(regime);
     if (regime == 6) return fill_neutral_run(op, dt, nseg, out, out_idx, st);
     return dispatch<SegRun>(op, dt, regime, in, nseg, L, out, out_idx, ws, st);
 }

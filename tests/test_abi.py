@@ -208,11 +208,15 @@ def test_workspace_queries_and_regimes(fs):
     assert r(1 << 13, 1 << 15) == 2
     assert r(4, 1 << 26) == 3 and r(1, 1 << 28) == 3
     assert r(64, 64, layout="col") == 4
-    assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 5
-    assert r(1 << 20, 3, scan=True) == 8 and r(1 << 20, 33, scan=True) == 5 and r(64, 7, scan=True, op="argmin") == 5
-    assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 5  # KS2: >= 4 rows per SM
-    assert r(1 << 12, 2048, scan=True) == 5 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 9
-    assert r(1 << 20, 512, scan=True, dtype=torch.int64) == 7 and r(1 << 20, 1024, scan=True, dtype=torch.int64) == 5
+    assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 11
+    assert r(1 << 20, 3, scan=True) == 8 and r(1 << 20, 33, scan=True) == 11 and r(64, 7, scan=True, op="argmin") == 5
+    assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 11  # KS2: >= 1 row per SM
+    assert r(64, 16384, scan=True, op="argmin") == 5 and r(64, 16385, scan=True) == 5
+    assert r(1 << 12, 2048, scan=True) == 10 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 10
+    assert r(1 << 12, 8192, scan=True) == 10 and r(1 << 12, 16384, scan=True, dtype=torch.int64) == 9
+    assert r(1 << 20, 512, scan=True, dtype=torch.int64) == 7 and r(1 << 20, 1024, scan=True, dtype=torch.int64) == 10
+    assert r(1, 1 << 28, scan=True) == 12 and r(2, 1 << 27, scan=True) == 12 and r(1, 5, scan=True) == 12
+    assert r(4096, 1000, scan=True, op="argmin") == 5 and r(1 << 21, 128, scan=True, op="argmin") == 7
     assert r(0, 64) == 6 and r(64, 0) == 6
     assert r(64, 64, dtype=torch.int64, op="argmin") == 0
     fs.force_seg_regime(2)
@@ -221,8 +225,22 @@ def test_workspace_queries_and_regimes(fs):
     finally:
         fs.force_seg_regime(-1)
     assert r(1 << 20, 16) == 0
-    with pytest.raises(fs.FutsegError):
-        fs.force_seg_regime(9)
+    for forced, shape, want in ((5, (1 << 20, 1024), 5), (12, (1 << 10, 1024), 12), (11, (1 << 10, 1024), 11),
+                                (12, (1 << 20, 3), 8), (11, (64, 63), 11), (9, (1 << 12, 2048), 10)):
+        fs.force_seg_regime(forced)
+        try:
+            assert r(*shape, scan=True) == want, (forced, shape)
+        finally:
+            fs.force_seg_regime(-1)
+    fs.force_seg_regime(5)
+    try:
+        assert r(64, 63, scan=True, op="argmin") == 5
+    finally:
+        fs.force_seg_regime(-1)
+    for bad in (-2, 4, 6, 13):
+        with pytest.raises(fs.FutsegError):
+            fs.force_seg_regime(bad)
+    assert fs.last_seg_regime() == -1  # no segmented call has run in this (CPU-only) process
 
 
 def test_python_layer_refuses_cpu_tensors(fs):

@@ -523,8 +523,10 @@ def test_seg_scan_few_long_rows(fs):
 
 @pytest.mark.parametrize("seglen", [4, 64, 512])
 def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
-    """KS0 needs 16-byte aligned buffers: a misaligned view takes the look-back scan and
-    still matches the oracle."""
+    """KS0 needs 16-byte aligned buffers: a misaligned view of power-of-two rows falls back
+    -- to KS1 / KS3 (element-aligned shared-memory staging) for add/min/max at L = 4 / 64,
+    512, to the segmented look-back scan for argmin -- and still matches the oracle
+    (test_gpu_edges forces the look-back scan for every op and dtype)."""
     nseg = 777
     for dt, op in ((np.float32, "add"), (np.int32, "max"), (np.float32, "argmin")):
         x = workloads.mixed(nseg * seglen, seglen, dt)

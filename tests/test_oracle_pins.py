@@ -517,3 +517,23 @@ def test_redomap_is_reduce_of_map():
     d = oracle.nn_dist(lat, lng, *q)
     assert oracle.redomap(lat, "min", "nn_dist", lng, q) == d.min()
     np.testing.assert_array_equal(oracle.scanomap(lat, "max", "nn_dist", lng, q), np.maximum.accumulate(d))
+
+
+def _r18_fixture():
+    g = gold("kmeans_r18_fma.json")
+    pts = np.array([[float.fromhex(v) for v in row] for row in g["points"]], np.float32)
+    cen = np.array([[float.fromhex(v) for v in row] for row in g["centres"]], np.float32)
+    return g, pts, cen
+
+
+def test_golden_kmeans_r18_fma_rounding():
+    """Reading R18 pinned: points whose R18 membership (exact rationals, one rounding per
+    fma, index order, first centre on ties; tools/gen_golden_r18.py) differs from the
+    decision under separately rounded mul+add, reversed order, exact real arithmetic, an f64
+    accumulator, or last-wins ties.  An oracle making any of those mistakes fails here."""
+    g, pts, cen = _r18_fixture()
+    assert set(g["discriminates"]) == {"mul_add", "reversed", "exact", "f64_acc", "le_ties"}
+    m, _, counts, _, _ = oracle.kmeans_step(pts, cen)
+    bad = [(i, w) for i, (a, b, w) in enumerate(zip(m.tolist(), g["membership"], g["discriminates"])) if a != b]
+    assert not bad, bad
+    assert counts[2] == 0
