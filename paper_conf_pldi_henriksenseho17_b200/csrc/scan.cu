@@ -1438,7 +1438,9 @@ template <int OP, typename T> struct ScanRun {
                     const int64_t nseg = n / L;
                     const int64_t R = L >= kRowsElems ? 1 : kRowsElems / L;
                     const int smem = (int)(R * L * (int64_t)sizeof(T));
-                    if (smem > 48 * 1024)
+                    // (the kernel's static shared words count against the 48 KB default too:
+                    // L = 12288 f32 is exactly 48 KB dynamic)
+                    if (smem > 32 * 1024)
                         cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
                     int64_t grid = ceil_div(nseg, R);
                     const int64_t cap = resident_blocks((const void *)kr, 256, (size_t)smem);
@@ -1449,7 +1451,7 @@ template <int OP, typename T> struct ScanRun {
                 if (rg == RG_KS1) {
                     auto kt = segscan_tile_kernel<OP, T>;
                     const int smem = (int)((256 * L + 256 * L / 32 + 1) * sizeof(T));
-                    if (smem > 48 * 1024)
+                    if (smem > 32 * 1024)
                         cudaFuncSetAttribute((const void *)kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
                     const int64_t nseg = n / L;
                     int64_t grid = ceil_div(nseg, 256);
