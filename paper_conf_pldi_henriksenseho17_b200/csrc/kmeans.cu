@@ -1,7 +1,7 @@
 // kmeans.cu -- NEXT-1: one fused iteration of Rodinia's K-means (Sec. 2.4,
 // L445-531; L1628-1649; fusion F6 L1075-1090: the assignment map is fused into the
-// stream_red that computes the new centres, so the membership array never has to be
-// re-read and the points are read once).
+// stream_red that computes the new centres, so the points are read once and the
+// membership array never has to be re-read).
 //
 //   membership[i] = argmin_c E(i, c), first c on ties            (readings R3, R18)
 //   E(i, c)       = sum_j (x_ij - c_cj)^2, f32, j in order, acc = fma(t, t, acc)
@@ -9,474 +9,704 @@
 //   new_centres   = sums / counts; an empty cluster keeps its centre     (R19)
 //   delta         = #{ i : membership[i] != prev[i] }  (Rodinia's convergence test)
 //
-// B200 design.  The distance computation is the one dense contraction on the path
-// ([n][d] points x [d][k] centres), so it runs on the tensor cores: warp-level
-// mma.sync m16n8k8 TF32 computes s = x . c for 16 rows x 32 centres per stage, and
-// d~_c = |c|^2 - 2 s ranks the centres (|x|^2 is the same for every centre).  TF32
-// is not the reading's f32 arithmetic, so the argmin is made EXACT by a bound: with
-// both operands rounded to TF32 (cvt.rna, 2^-11 relative each),
-//     | (E(i,c) - |x|^2) - d~_c |  <=  delta_c = 2^-9 (1 + 2^-7) |x| |c| + 2^-17 (|x| + |c|)^2
-// (input rounding of the 2 x.c term, plus the f32 rounding of E itself and of the
-// accumulation, generously).  Every centre with d~_c - delta_c <= min_c' (d~_c' +
-// delta_c') is a candidate; the true argmin of E is always one.  A row with one
-// candidate is decided; a row with several re-evaluates E exactly, in the reading's
-// f32 order, for its candidates only (CUDA cores, from the staged row).  Rows are
-// streamed through a per-warp TMA ring (as stream_red), the row norms come from the
-// A-fragment loads, and the decided keys feed the stream_red accumulation of the same
-// stage (lane-private shared-memory columns 0..31, cluster-owner registers for
-// columns 32..d-1).  Chunk results combine warp -> CTA -> last CTA, which also
-// divides by the counts.
+// B200 design: both contractions of the step run on the 5th-generation tensor cores
+// (tcgen05.mma kind::tf32, accumulators in TMEM); the CUDA cores stage operands and
+// take the per-row decision.  A stage is 128 consecutive points (one M = 128 tile); a
+// CTA per SM streams its contiguous chunk of stages; warps are specialised:
+//
+//   producer  (1 warp)  1-D TMA bulk copies of the stages' rows into an NR-slot ring.
+//   convert   (4 warps) thread r owns row r of a stage: reads it (conflict-free 8-byte
+//             loads), computes |x|^2, splits every x into hi = x with the low 13 mantissa
+//             bits cleared (exactly TF32) and lo = x - hi (exact), and writes
+//               - hi | 1 1 (columns d, d+1) and lo into TMEM (tcgen05.st, TMEM lane r),
+//                 the K-major A operand of MMA1, plus |x|^2 in one more column;
+//               - hi[0..31], lo[0..31] and the extras (hi/lo of columns 32.., a 1.0 for
+//                 the count) into shared memory as the MN-major A operand of MMA2
+//                 (128B swizzle with 32-byte atoms: the layout tf32 MN-major needs).
+//   MMA       (1 thread) MMA1: d~ = |c|^2 - 2 x.c for 128 rows x NC centres as three
+//             TF32 products (hi.Bhi + hi.Blo + lo.Bhi; B = -2c split the same way, |c|^2
+//             split in the augmented columns) -> TMEM D1.  MMA2: D2[j][c] += sum over the
+//             stage's rows of X[row][j] * onehot[row][c] -> TMEM D2, 16 stages per buffer
+//             (double-buffered).  It polls both queues so MMA1 runs ahead of decisions.
+//   decide    (4 warps) thread r: one tcgen05.ld of its NC values, minimum m, candidates
+//             d~_c <= m + 2 delta(x).  delta bounds |d~_c - (E_f32(x, c) - |x|^2)| (TF32
+//             splitting 6 * 2^-20 |x||c|, the f32 |c|^2, the tensor core's f32
+//             accumulation and the f32 rounding of R18's own E: all below 2^-15 (|x| +
+//             |c|)^2 <= 2^-14 (|x|^2 + max|c|^2)), so R18's argmin is always a
+//             candidate.  One candidate decides the row; several (rare) are re-evaluated
+//             in R18's exact f32 order from x = hi + lo.  Writes the one-hot B operand of
+//             MMA2 (K-major, one 1.0 per row, reset when the slot comes back),
+//             membership and delta; every 16 stages moves D2 into registers (two-level
+//             f32 accumulation).
+// Chunk results combine CTA -> workspace -> last CTA, which divides by the counts.
+#include <cuda_bf16.h>
+#include <stdlib.h>
+
 #include "internal.cuh"
 
 namespace fs {
 
-constexpr int kKmThreads = 256;
-constexpr int kKmWarps = kKmThreads / 32;
-constexpr int kKmRS = 16;      // rows per stage = one m16 tile
-constexpr int kKmStages = 2;
-constexpr int kKmK = 32;       // max clusters (4 n-tiles of 8)
-constexpr int kKmNT = kKmK / 8;
-constexpr int kKmMaxD = 40;    // 5 k-steps of 8
-constexpr int kKmXR = kKmMaxD - 32;  // extra columns (32..d-1) held by the cluster-owner lane
-constexpr int kKmPairs = 128;        // per-warp scratch of (row, candidate) pairs for exact re-evaluation
+constexpr int kKmRows = 128;   // rows per stage (UMMA M)
+constexpr int kKmRing = 5;     // TMA ring slots (at most)
+constexpr int kKmCv = 2;       // convert groups of 4 warps; group g converts stages s = g (mod 2)
+constexpr int kKmNA = 3;       // TMEM stage slots (A operand, |x|^2, D1)
+constexpr int kKmNXMax = 4;    // shared-memory stage slots (MMA2 operands), at most
+constexpr int kKmThreads = (4 * kKmCv + 4 + 2) * 32;  // convert + decide + producer + MMA warp
+constexpr int kKmWarpDecide = 4 * kKmCv, kKmWarpProd = 4 * kKmCv + 4, kKmWarpMma = 4 * kKmCv + 5;
+constexpr int kKmK = 32;       // max clusters
+constexpr int kKmMaxD = 40;
+constexpr int kKmSeg = 16;     // stages per D2 buffer
 
-__device__ __forceinline__ uint32_t to_tf32(float x) {
-    uint32_t r;
-    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+__device__ __forceinline__ uint32_t km_smem(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void km_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(km_smem(bar)) : "memory");
+}
+__device__ __forceinline__ void km_wait(uint64_t *bar, unsigned parity) {  // suspends in hardware while waiting
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(km_smem(bar)), "r"(parity)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+// no-swizzle UMMA shared-memory descriptor: start, leading (LBO) and stride (SBO) byte
+// offsets >> 4, version 1 (sm_100), layout type 0 (SWIZZLE_NONE)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
+}
+// instruction descriptor, kind::f16 with bf16 A/B and f32 D, M = 128, N, majors (0 K, 1 MN)
+__host__ __device__ constexpr uint32_t umma_idesc_bf16(int N, int a_mn, int b_mn) {
+    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
+           ((uint32_t)(N >> 3) << 17) | ((uint32_t)(kKmRows >> 4) << 24);
+}
+// D[tmem] (+)= A[smem] . B[smem]
+__device__ __forceinline__ void umma_bf16_ss(uint32_t dtmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(dtmem),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+}
+// D[tmem] (+)= A[tmem] (K-major) . B[smem]
+__device__ __forceinline__ void umma_bf16_ts(uint32_t dtmem, uint32_t atmem, uint64_t b, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(dtmem),
+        "r"(atmem), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+}
+__device__ __forceinline__ void umma_commit(uint64_t *bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(km_smem(bar))
+                 : "memory");
+}
+// 32 lanes x 32 consecutive 32-bit columns: thread i of the warp gets lane (base + i)
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+    uint32_t r[32];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+          "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+          "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr)
+        : "memory");
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void km_tma_load(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     km_smem(dst)),
+                 "l"(src), "r"(bytes), "r"(km_smem(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void km_bar_sync(int id, int count) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+__device__ __forceinline__ uint32_t bf2(float lo, float hi) {  // packed bf16 pair, round to nearest even
+    const __nv_bfloat162 p = __floats2bfloat162_rn(lo, hi);
+    return *reinterpret_cast<const uint32_t *>(&p);
+}
+__device__ __forceinline__ float bfr(float x) { return __bfloat162float(__float2bfloat16_rn(x)); }
+__device__ __forceinline__ float fmin3(float a, float b, float c) {
+    float r;
+    asm("min.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
     return r;
 }
-
-__device__ __forceinline__ void mma_tf32(float (&c)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
-                                         uint32_t b0, uint32_t b1) {
-    asm volatile(
-        "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-        "{%0,%1,%2,%3};"
-        : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
-        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+__device__ __forceinline__ void tmem_ld64(uint32_t taddr, float (&v)[64]) {
+    float a[32], b[32];
+    tmem_ld32(taddr, a);
+    tmem_ld32(taddr + 32, b);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+        v[i] = a[i];
+        v[32 + i] = b[i];
+    }
 }
-
-struct KmShared {  // per-CTA, after the per-warp regions
-    float cen[kKmK * kKmMaxD];  // centres (f32, as given), rows >= k unused
-    float csq[kKmK];            // |c|^2 (+inf for padding centres)
-    float cn[kKmK];             // |c|
-};
-
-// E(x, c) exactly as reading R18 / the oracle: f32, j in order, one rounding per fma.
+__device__ __forceinline__ bool km_test(uint64_t *bar, unsigned parity) {
+    uint32_t done;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(km_smem(bar)), "r"(parity)
+        : "memory");
+    return done != 0;
+}
+__device__ __forceinline__ void tmem_st8u(uint32_t taddr, const uint32_t (&v)[8]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), "r"(v[0]),
+                 "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+                 : "memory");
+}
+__device__ __forceinline__ void tmem_st1(uint32_t taddr, float v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(__float_as_uint(v)) : "memory");
+}
+__device__ __forceinline__ float tmem_ld1(uint32_t taddr) {
+    uint32_t r;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%1];" : "=r"(r) : "r"(taddr) : "memory");
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+    return __uint_as_float(r);
+}
+// E(x, c) exactly as reading R18 / the oracle: f32, j in order, one rounding per fma
 __device__ __forceinline__ float km_exact(const float *x, const float *c, int d) {
     float acc = 0.f;
     for (int j = 0; j < d; ++j) {
-        const float t = __fsub_rn(x[j], c[j]);
-        acc = __fmaf_rn(t, t, acc);
+        const float tt = __fsub_rn(__ldg(x + j), c[j]);
+        acc = __fmaf_rn(tt, tt, acc);
     }
     return acc;
 }
 
-template <int KS, int XR>
-__global__ void __launch_bounds__(kKmThreads, 2)
-kmeans_step_kernel(const float *__restrict__ pts, int64_t n, int d, const float *__restrict__ cen, int k,
-                   const int32_t *__restrict__ prev, int32_t *__restrict__ membership, int64_t rows_per_warp,
-                   float *partials, int *pcounts, unsigned *ticket, unsigned long long *gdelta, float *sums,
-                   int32_t *counts, float *new_cen, int64_t *delta_out) {
-    extern __shared__ __align__(128) unsigned char smem[];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int g = lane >> 2, t = lane & 3;
-    const int XW = d > 32 ? d - 32 : 0;
-    const unsigned vbytes = (unsigned)(kKmRS * d * 4);
-    const unsigned slot = vbytes + kKmRS * 4;
-    const size_t warp_bytes = (size_t)kKmStages * slot + kKmStages * 8 + (size_t)(kKmK + 1) * 32 * 4 + kKmPairs * 8;
-    unsigned char *wbase = smem + (size_t)warp * warp_bytes;
-    unsigned char *ring = wbase;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(wbase + kKmStages * slot);
-    float *s_acc = reinterpret_cast<float *>(wbase + kKmStages * slot + kKmStages * 8);  // [K+1][32]
-    unsigned *s_pair = reinterpret_cast<unsigned *>(s_acc + (kKmK + 1) * 32);          // [kKmPairs]
-    float *s_e = reinterpret_cast<float *>(s_pair + kKmPairs);                          // [kKmPairs]
-    KmShared &sh = *reinterpret_cast<KmShared *>(smem + (size_t)kKmWarps * warp_bytes);
 
-    // ---- centres: shared copy, norms, TF32 B fragments (k permuted: logical t <-> column 2t,
-    //      logical t+4 <-> column 2t+1 of each 8-column block, so A loads are column pairs)
-    for (int e = threadIdx.x; e < kKmK * kKmMaxD; e += kKmThreads) {
-        const int c = e / kKmMaxD, j = e - c * kKmMaxD;
-        sh.cen[e] = (c < k && j < d) ? cen[c * d + j] : 0.f;
+
+struct KmBars {
+    uint64_t raw_full[kKmRing], raw_empty[kKmRing];
+    uint64_t a1full[kKmNA], d1full[kKmNA], slotfree[kKmNA];
+    uint64_t ohfull[kKmNXMax], x2free[kKmNXMax];
+    uint64_t d2full[2], d2free[2];
+    uint32_t tmem_base;
+    float cmax2;
+};
+
+// Operand geometry for a given d (host and device):
+//   KP  = bf16 columns of one A piece: d + 3 augmentation columns, padded to 16
+//   JB  = first MMA2 row of the a2 piece (a1 rows 0..d-1, the count row d), padded to 8
+//   NG  = MMA2 M-groups written (8 rows each): JB/8 + ceil(d/8)
+struct KmGeom {
+    int KP, JB, NG;
+    __host__ __device__ KmGeom(int d) : KP((d + 3 + 15) / 16 * 16), JB((d + 1 + 7) / 8 * 8), NG(0) {
+        NG = JB / 8 + (d + 7) / 8;
     }
-    __syncthreads();
-    if (threadIdx.x < kKmK) {
-        const int c = threadIdx.x;
-        float s = 0.f;
-        for (int j = 0; j < d; ++j) s = __fmaf_rn(sh.cen[c * kKmMaxD + j], sh.cen[c * kKmMaxD + j], s);
-        sh.csq[c] = c < k ? s : __int_as_float(0x7f800000);
-        sh.cn[c] = c < k ? sqrtf(s) : 0.f;
-    }
-    for (int e = lane; e < (kKmK + 1) * 32; e += 32) s_acc[e] = 0.f;
-    uint32_t bf[kKmNT][KS][2];
+    __host__ __device__ int x2_bytes() const { return 16 * NG * 128; }
+};
+
+__device__ __forceinline__ uint32_t cvt_bf2(float lo, float hi) {  // packed bf16 pair, round to nearest even
+    uint32_t r;
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+    return r;
+}
+
+// One row of a stage -> the two bf16 pieces of every column, written as the MMA1 A operand (TMEM
+// lane of the calling thread, K-major pairs: [a1 | 1 1 1 | 0..] then [a2 | 0..], KP columns each)
+// and as the MMA2 A operand (shared memory, MN-major: the row is the K index, a1 rows 0..d-1, the
+// count row d, a2 rows JB..JB+d-1).  Returns |x|^2 (f32).
+template <bool FULL, bool EVEN>
+__device__ __forceinline__ float km_convert_row(const float *src, int d, bool valid, const KmGeom &G, int qd,
+                                                uint32_t ta, unsigned char *xr) {
+    float nrm = 0.f;
 #pragma unroll
-    for (int nt = 0; nt < kKmNT; ++nt)
+    for (int q = 0; q < 3; ++q) {  // 16 columns per chunk (KP <= 48)
+        if (16 * q < G.KP) {
+            uint32_t w1[8], w2[8];
+            const bool tail = q >= qd;  // the chunk holding column d (augmentation, count)
 #pragma unroll
-        for (int ks = 0; ks < KS; ++ks) {
-            const float *cr = sh.cen + (nt * 8 + g) * kKmMaxD + ks * 8 + 2 * t;
-            bf[nt][ks][0] = to_tf32(cr[0]);
-            bf[nt][ks][1] = to_tf32(cr[1]);
+            for (int t = 0; t < 8; ++t) {
+                const int j0 = 16 * q + 2 * t, j1 = j0 + 1;
+                float x0, x1;
+                if (EVEN && (!tail || j1 < d)) {
+                    const float2 p2 = *reinterpret_cast<const float2 *>(src + j0);
+                    x0 = p2.x;
+                    x1 = p2.y;
+                } else if (!tail) {
+                    x0 = src[j0];
+                    x1 = src[j1];
+                } else {
+                    x0 = j0 < d ? src[j0] : 0.f;
+                    x1 = j1 < d ? src[j1] : 0.f;
+                }
+                if (!FULL && !valid) x0 = x1 = 0.f;
+                nrm = __fmaf_rn(x0, x0, nrm);
+                nrm = __fmaf_rn(x1, x1, nrm);
+                w1[t] = cvt_bf2(x0, x1);
+                w2[t] = cvt_bf2(__fsub_rn(x0, __uint_as_float(w1[t] << 16)),
+                                __fsub_rn(x1, __uint_as_float(w1[t] & 0xFFFF0000u)));
+            }
+            uint32_t wt[8], wx[8];
+#pragma unroll
+            for (int t = 0; t < 8; ++t) {
+                wt[t] = w1[t];
+                wx[t] = w1[t];
+            }
+            if (tail) {  // MMA1 A: 1.0 in columns d, d+1, d+2; MMA2 A: the count at d
+#pragma unroll
+                for (int t = 0; t < 8; ++t) {
+                    const int j0 = 16 * q + 2 * t, j1 = j0 + 1;
+                    wt[t] |= ((j0 >= d && j0 <= d + 2) ? 0x3F80u : 0u) | ((j1 >= d && j1 <= d + 2) ? 0x3F800000u : 0u);
+                    wx[t] |= ((j0 == d && valid) ? 0x3F80u : 0u) | ((j1 == d && valid) ? 0x3F800000u : 0u);
+                }
+            }
+            tmem_st8u(ta + 8 * q, wt);
+            tmem_st8u(ta + G.KP / 2 + 8 * q, w2);
+            if (16 * q < G.JB) *reinterpret_cast<uint4 *>(xr + (2 * q) * 128) = make_uint4(wx[0], wx[1], wx[2], wx[3]);
+            if (16 * q + 8 < G.JB)
+                *reinterpret_cast<uint4 *>(xr + (2 * q + 1) * 128) = make_uint4(wx[4], wx[5], wx[6], wx[7]);
+            if (16 * q < d)
+                *reinterpret_cast<uint4 *>(xr + (G.JB / 8 + 2 * q) * 128) = make_uint4(w2[0], w2[1], w2[2], w2[3]);
+            if (16 * q + 8 < d)
+                *reinterpret_cast<uint4 *>(xr + (G.JB / 8 + 2 * q + 1) * 128) = make_uint4(w2[4], w2[5], w2[6], w2[7]);
         }
-    __syncthreads();
-    // this thread's 8 centres (2 per n-tile): norms for the bound
-    float ccsq[kKmNT][2], cmax = 0.f;
-#pragma unroll
-    for (int nt = 0; nt < kKmNT; ++nt)
-#pragma unroll
-        for (int h = 0; h < 2; ++h) ccsq[nt][h] = sh.csq[nt * 8 + 2 * t + h];
-    for (int cc = 0; cc < k; ++cc) cmax = fmaxf(cmax, sh.cn[cc]);
-    cmax *= 1.0001f;
+    }
+    return nrm;
+}
 
-    const int64_t gw = (int64_t)blockIdx.x * kKmWarps + warp;
-    const int64_t i0 = gw * rows_per_warp;
-    const int64_t i1 = i0 + rows_per_warp < n ? i0 + rows_per_warp : n;
-    const int64_t nfull = i1 > i0 ? (i1 - i0) / kKmRS : 0;
-    const int nst = (int)nfull + ((i1 > i0 && (i1 - i0) % kKmRS) ? 1 : 0);  // + one partial stage
-    if (lane == 0) {
-#pragma unroll
-        for (int s = 0; s < kKmStages; ++s) mbar_init(bars + s, 1);
+template <int NC, int DT>
+__global__ void __launch_bounds__(kKmThreads, 1)
+kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int NX, const float *__restrict__ cen,
+                 int k, const int32_t *__restrict__ prev, int32_t *__restrict__ membership, int64_t rows_per_cta,
+                 float *partials, int *pcounts, unsigned *ticket, unsigned long long *gdelta, float *sums,
+                 int32_t *counts, float *new_cen, int64_t *delta_out) {
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    unsigned char *smem =
+        reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int d = DT > 0 ? DT : d_rt;  // DT > 0: the width is a compile-time constant (C3 / C5: 34)
+    constexpr bool EVEN = DT > 0 && DT % 2 == 0;
+    const KmGeom G(d);
+    constexpr int N1 = 2 * NC;  // MMA1 N: (centre, b piece)
+    // ---- shared memory carve-up
+    const uint32_t raw_bytes = (uint32_t)(kKmRows * d * 4);
+    const uint32_t raw_slot = (raw_bytes + 1023u) & ~1023u;
+    const uint32_t x2_bytes = (uint32_t)G.x2_bytes();
+    constexpr uint32_t oh_bytes = NC / 8 * 2048;           // [centre group][16 row chunks][8 x 16 B]
+    const uint32_t LB2 = (uint32_t)(G.NG * 128);           // MMA2 A: K-group (8 rows) stride
+    const uint32_t SB1 = (uint32_t)(2 * G.KP / 8 * 128);  // MMA1 B: n-group stride (K1 = 2 KP)
+    unsigned char *raw = smem;                              // [NR][raw_slot]
+    unsigned char *x2 = raw + NR * raw_slot;                // [NX][x2_bytes] + 1 KB (MMA2 M read-beyond)
+    unsigned char *oh = x2 + NX * x2_bytes + 1024;          // [NX][oh_bytes]
+    unsigned char *b1 = oh + NX * oh_bytes;                 // [N1/8][K1/8][8 x 16 B]
+    float *cen_s = reinterpret_cast<float *>(b1 + (N1 / 8) * SB1);  // [NC][kKmMaxD]
+    KmBars &B = *reinterpret_cast<KmBars *>(cen_s + NC * kKmMaxD);
+
+    const int64_t i0 = (int64_t)blockIdx.x * rows_per_cta;
+    const int64_t i1 = i0 + rows_per_cta < n ? i0 + rows_per_cta : n;
+    const int64_t nrows = i1 > i0 ? i1 - i0 : 0;
+    const int nfull = (int)(nrows / kKmRows);
+    const int ns = nfull + ((nrows % kKmRows) ? 1 : 0);
+    const int nseg2 = (ns + kKmSeg - 1) / kKmSeg;
+
+    // ---- setup: barriers, TMEM, centre operand, zeroed MMA2 operands
+    if (tid == 0) {
+        for (int s = 0; s < NR; ++s) {
+            mbar_init(&B.raw_full[s], 1);
+            mbar_init(&B.raw_empty[s], 4);
+        }
+        for (int s = 0; s < kKmNA; ++s) {
+            mbar_init(&B.a1full[s], 4);
+            mbar_init(&B.d1full[s], 1);
+            mbar_init(&B.slotfree[s], 4);
+        }
+        for (int s = 0; s < NX; ++s) {
+            mbar_init(&B.ohfull[s], 4);
+            mbar_init(&B.x2free[s], 1);
+        }
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(&B.d2full[s], 1);
+            mbar_init(&B.d2free[s], 4);
+        }
         fence_mbar_init();
-        for (int s = 0; s < kKmStages && s < nfull; ++s) {
-            mbar_expect_tx(bars + s, vbytes);
-            tma_load_1d(ring + s * slot, pts + (i0 + (int64_t)s * kKmRS) * d, vbytes, bars + s);
-        }
     }
-    __syncwarp();
-    float xa[XR > 0 ? XR : 1];
-#pragma unroll
-    for (int e = 0; e < (XR > 0 ? XR : 1); ++e) xa[e] = 0.f;
-    unsigned wcnt = 0, wdelta = 0;
-    int s = 0;
-    unsigned phase = 0;
-    constexpr float kE1 = 1.0f / 512.0f * (1.0f + 1.0f / 128.0f), kE2 = 1.0f / 131072.0f;
-    for (int c = 0; c < nst; ++c) {
-        const int64_t r0 = i0 + (int64_t)c * kKmRS;
-        const bool full = c < nfull;
-        const int nv = full ? kKmRS : (int)(i1 - r0);
-        float *sv = reinterpret_cast<float *>(ring + s * slot);
-        int *sk = reinterpret_cast<int *>(ring + s * slot + vbytes);
-        if (full) {
-            mbar_wait(bars + s, phase);
-        } else {  // ragged tail of the chunk: plain loads into the (idle) slot, zero padding
-            for (int e = lane; e < kKmRS * d; e += 32) sv[e] = e < nv * d ? __ldg(pts + r0 * d + e) : 0.f;
+    if (warp == kKmWarpMma) {  // the MMA warp owns the TMEM allocation
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(km_smem(&B.tmem_base)),
+                     "r"(512)
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    for (int e = tid; e < NC * kKmMaxD; e += kKmThreads) {
+        const int c = e / kKmMaxD, j = e - c * kKmMaxD;
+        cen_s[e] = (c < k && j < d) ? cen[c * d + j] : 0.f;
+    }
+    for (int e = tid; e < (int)((NX * (x2_bytes + oh_bytes) + 1024) / 16); e += kKmThreads)
+        reinterpret_cast<uint4 *>(x2)[e] = make_uint4(0u, 0u, 0u, 0u);
+    __syncthreads();
+    // B1[n][k], K-major no swizzle: n < NC is centre n with the b1 piece of -2c and the |c|^2
+    // pieces q1 q2 q3 in columns d, d+1, d+2 of the a1 half; n >= NC is centre n - NC with the b2
+    // piece.  The a2 half of K (k >= KP) repeats the b piece without |c|^2.  Padding centres have
+    // |c|^2 = 2^100 (finite: 0 * it stays 0), so they are never candidates.
+    for (int e = tid; e < N1 * 2 * G.KP; e += kKmThreads) {
+        const int nn = e / (2 * G.KP), kk = e - nn * (2 * G.KP);
+        const int c = nn < NC ? nn : nn - NC, piece = nn < NC ? 0 : 1, j = kk < G.KP ? kk : kk - G.KP;
+        float v = 0.f;
+        if (j < d) {
+            const float b = c < k ? -2.f * cen_s[c * kKmMaxD + j] : 0.f;
+            const float p1 = bfr(b);
+            v = piece == 0 ? p1 : bfr(__fsub_rn(b, p1));
+        } else if (kk < G.KP && piece == 0 && j <= d + 2) {
+            float c2 = 0x1p100f;
+            if (c < k) {
+                double sq = 0.0;
+                for (int q = 0; q < d; ++q) sq += (double)cen_s[c * kKmMaxD + q] * (double)cen_s[c * kKmMaxD + q];
+                c2 = (float)sq;
+            }
+            const float q1 = bfr(c2), q2 = bfr(__fsub_rn(c2, q1)), q3 = bfr(__fsub_rn(__fsub_rn(c2, q1), q2));
+            v = j == d ? q1 : (j == d + 1 ? q2 : q3);
+        }
+        *reinterpret_cast<__nv_bfloat16 *>(b1 + (nn >> 3) * SB1 + (kk >> 3) * 128 + (nn & 7) * 16 + (kk & 7) * 2) =
+            __float2bfloat16_rn(v);
+    }
+    if (tid < 32) {
+        float m = 0.f;
+        for (int c = lane; c < k; c += 32) {
+            float sq = 0.f;
+            for (int q = 0; q < d; ++q) sq = __fmaf_rn(cen_s[c * kKmMaxD + q], cen_s[c * kKmMaxD + q], sq);
+            m = fmaxf(m, sq);
+        }
+        for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        if (lane == 0) B.cmax2 = m * 1.0001f;
+    }
+    fence_proxy_async();  // operands written by threads: visible to the tensor core
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = B.tmem_base;
+    // TMEM columns: D1 slots [0, NA N1), D2 buffers (2 NC), |x|^2 (32), A slots (KP each)
+    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tN = tD2 + 2 * NC, tA = tN + 32;
+
+    float *s_part = reinterpret_cast<float *>(x2);  // [128][NC] CTA partial (after the loop)
+    if (warp < kKmWarpDecide) {
+        // =============================== convert: row r -> bf16 pieces a1 = bf16(x), a2 = bf16(x - a1)
+        // (x = a1 + a2 + O(2^-18 |x|)) in TMEM (MMA1 A, K-major) and shared memory (MMA2 A, MN-major)
+        const int g = warp >> 2, wl = warp & 3, r = wl * 32 + lane;
+        const uint32_t t_lane = (uint32_t)(wl * 32) << 16;
+        const int qd = d >> 4;  // chunks of 16 columns that hold only data
+        for (int s = g; s < ns; s += kKmCv) {
+            const int64_t r0 = i0 + (int64_t)s * kKmRows;
+            const bool full = s < nfull;
+            const int nv = full ? kKmRows : (int)(i1 - r0);
+            const bool valid = r < nv;
+            const float *src;
+            if (full) {
+                km_wait(&B.raw_full[s % NR], (unsigned)((s / NR) & 1));
+                src = reinterpret_cast<const float *>(raw + (s % NR) * raw_slot) + (size_t)r * d;
+            } else {
+                src = pts + (r0 + (valid ? r : 0)) * d;
+            }
+            const int sa = s % kKmNA, sx = s % NX;
+            if (s >= kKmNA) km_wait(&B.slotfree[sa], (unsigned)(((s / kKmNA) - 1) & 1));  // decide read D1
+            if (s >= NX) km_wait(&B.x2free[sx], (unsigned)(((s / NX) - 1) & 1));         // MMA2 read X
+            tc_fence_after();
+            const uint32_t ta = tA + t_lane + (uint32_t)(sa * G.KP);
+            unsigned char *xr = x2 + sx * x2_bytes + (r >> 3) * LB2 + (r & 7) * 16;
+            float nrm;
+            if (full)
+                nrm = km_convert_row<true, EVEN>(src, d, true, G, qd, ta, xr);
+            else
+                nrm = km_convert_row<false, EVEN>(src, d, valid, G, qd, ta, xr);
+            tmem_st1(tN + t_lane + (uint32_t)sa, nrm);
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+            fence_proxy_async();
+            tc_fence_before();
             __syncwarp();
+            if (lane == 0) {
+                if (full) km_arrive(&B.raw_empty[s % NR]);
+                km_arrive(&B.a1full[sa]);
+            }
         }
-        // ---- assignment: s = x . c on the tensor cores, row norms from the same loads
-        float acc[kKmNT][4];
+    } else if (warp < kKmWarpProd) {
+        // =============================== decide: candidates from the tensor-core ranking, exact R18
+        // for near-ties; one-hot MMA2 operand; membership; delta; D2 buffers -> registers
+        const int wl = warp - kKmWarpDecide, r = wl * 32 + lane;
+        const uint32_t t_lane = (uint32_t)(wl * 32) << 16;
+        const float cmax2 = B.cmax2;
+        float acc_tot[NC];
 #pragma unroll
-        for (int nt = 0; nt < kKmNT; ++nt) acc[nt][0] = acc[nt][1] = acc[nt][2] = acc[nt][3] = 0.f;
-        float nx0 = 0.f, nx1 = 0.f;
+        for (int c = 0; c < NC; ++c) acc_tot[c] = 0.f;
+        int ohpos[kKmNXMax];
 #pragma unroll
-        for (int ks = 0; ks < KS; ++ks) {
-            const int c0 = ks * 8 + 2 * t;
-            const float x00 = c0 < d ? sv[g * d + c0] : 0.f, x01 = c0 + 1 < d ? sv[g * d + c0 + 1] : 0.f;
-            const float x10 = c0 < d ? sv[(g + 8) * d + c0] : 0.f, x11 = c0 + 1 < d ? sv[(g + 8) * d + c0 + 1] : 0.f;
-            nx0 = __fmaf_rn(x00, x00, __fmaf_rn(x01, x01, nx0));
-            nx1 = __fmaf_rn(x10, x10, __fmaf_rn(x11, x11, nx1));
-            const uint32_t a0 = to_tf32(x00), a1 = to_tf32(x10), a2 = to_tf32(x01), a3 = to_tf32(x11);
+        for (int q = 0; q < kKmNXMax; ++q) ohpos[q] = -1;
+        unsigned wdelta = 0;
+        int flushed = 0;
+        auto flush = [&]() {
+            const int b2 = flushed & 1;
+            km_wait(&B.d2full[b2], (unsigned)((flushed >> 1) & 1));
+            tc_fence_after();
+            float v[32];
+            tmem_ld32(tD2 + t_lane + (uint32_t)(b2 * NC), v);
 #pragma unroll
-            for (int nt = 0; nt < kKmNT; ++nt) mma_tf32(acc[nt], a0, a1, a2, a3, bf[nt][ks][0], bf[nt][ks][1]);
-        }
-        nx0 += __shfl_xor_sync(0xffffffffu, nx0, 1);
-        nx0 += __shfl_xor_sync(0xffffffffu, nx0, 2);
-        nx1 += __shfl_xor_sync(0xffffffffu, nx1, 1);
-        nx1 += __shfl_xor_sync(0xffffffffu, nx1, 2);
-        nx0 = sqrtf(nx0) * 1.0001f;  // |x| (an upper bound up to f32 rounding)
-        nx1 = sqrtf(nx1) * 1.0001f;
-        // d~ = |c|^2 - 2 s for rows g, g+8 and centres 8nt + 2t + h; one bound per row with
-        // the largest centre norm: candidates are d~_c <= min_c' d~_c' + 2 e(row)
-        const float e0 = kE1 * nx0 * cmax + kE2 * (nx0 + cmax) * (nx0 + cmax);
-        const float e1 = kE1 * nx1 * cmax + kE2 * (nx1 + cmax) * (nx1 + cmax);
-        float dd0[kKmNT][2], dd1[kKmNT][2];
-        float u0 = __int_as_float(0x7f800000), u1 = u0;
+            for (int c = 0; c < NC; ++c) acc_tot[c] = __fadd_rn(acc_tot[c], v[c]);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) km_arrive(&B.d2free[b2]);
+            ++flushed;
+        };
+        for (int s = 0; s < ns; ++s) {
+            const int64_t r0 = i0 + (int64_t)s * kKmRows;
+            const int nv = s < nfull ? kKmRows : (int)(i1 - r0);
+            const bool valid = r < nv;
+            const int sa = s % kKmNA, sx = s % NX;
+            const int pv = (prev && valid) ? __ldg(prev + r0 + r) : 0;  // in flight during the wait
+            km_wait(&B.d1full[sa], (unsigned)((s / kKmNA) & 1));
+            tc_fence_after();
+            float dd[NC];
+            {
+                float v[32];
+                tmem_ld32(tD1 + t_lane + (uint32_t)(sa * N1), v);
 #pragma unroll
-        for (int nt = 0; nt < kKmNT; ++nt)
+                for (int c = 0; c < NC; ++c) dd[c] = v[c];
+                if (NC == 32) {
+                    tmem_ld32(tD1 + t_lane + (uint32_t)(sa * N1 + 32), v);
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                dd0[nt][h] = __fmaf_rn(-2.f, acc[nt][h], ccsq[nt][h]);
-                dd1[nt][h] = __fmaf_rn(-2.f, acc[nt][2 + h], ccsq[nt][h]);
-                u0 = fminf(u0, dd0[nt][h]);
-                u1 = fminf(u1, dd1[nt][h]);
-            }
-        u0 = fminf(u0, __shfl_xor_sync(0xffffffffu, u0, 1));
-        u0 = fminf(u0, __shfl_xor_sync(0xffffffffu, u0, 2));
-        u1 = fminf(u1, __shfl_xor_sync(0xffffffffu, u1, 1));
-        u1 = fminf(u1, __shfl_xor_sync(0xffffffffu, u1, 2));
-        u0 += 2.f * e0;
-        u1 += 2.f * e1;
-        unsigned m0 = 0, m1 = 0;
+                    for (int c = 0; c < NC; ++c) dd[c] = __fadd_rn(dd[c], v[c]);
+                } else {
 #pragma unroll
-        for (int nt = 0; nt < kKmNT; ++nt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                m0 |= (dd0[nt][h] <= u0 ? 1u : 0u) << (nt * 8 + h);
-                m1 |= (dd1[nt][h] <= u1 ? 1u : 0u) << (nt * 8 + h);
-            }
-        m0 <<= 2 * t;  // this thread's centres are 8nt + 2t + h
-        m1 <<= 2 * t;
-        m0 |= __shfl_xor_sync(0xffffffffu, m0, 1);
-        m0 |= __shfl_xor_sync(0xffffffffu, m0, 2);
-        m1 |= __shfl_xor_sync(0xffffffffu, m1, 1);
-        m1 |= __shfl_xor_sync(0xffffffffu, m1, 2);
-        // lane r < 16 decides row r
-        const unsigned ma = __shfl_sync(0xffffffffu, m0, (lane & 7) * 4);
-        const unsigned mb = __shfl_sync(0xffffffffu, m1, (lane & 7) * 4);
-        const unsigned cm = lane < kKmRS ? (lane < 8 ? ma : mb) : 0u;
-        int key = __ffs(cm) - 1;
-        // rows with several candidates: E in the reading's exact f32 order, one (row,
-        // candidate) pair per lane -- all of the stage's pairs in one 34-step pass
-        const unsigned np = (cm & (cm - 1)) ? (unsigned)__popc(cm) : 0u;
-        if (__any_sync(0xffffffffu, np)) {
-            unsigned incl = np;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const unsigned v = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += v;
-            }
-            const unsigned total = __shfl_sync(0xffffffffu, incl, 31);
-            if (total <= (unsigned)kKmPairs) {
-                unsigned off = incl - np;
-                for (unsigned b = np ? cm : 0u; b; b &= b - 1) s_pair[off++] = (lane << 8) | (__ffs(b) - 1);
-                __syncwarp();
-                for (unsigned p = lane; p < total; p += 32) {
-                    const unsigned pr = s_pair[p];
-                    s_e[p] = km_exact(sv + (pr >> 8) * d, sh.cen + (pr & 255) * kKmMaxD, d);
+                    for (int c = 0; c < NC; ++c) dd[c] = __fadd_rn(dd[c], v[NC + c]);
                 }
-                __syncwarp();
-                if (np) {  // pairs are in ascending centre order: strict < keeps the first on ties
-                    const unsigned o0 = incl - np;
-                    float best = s_e[o0];
-                    key = (int)(s_pair[o0] & 255);
-                    for (unsigned p = o0 + 1; p < incl; ++p)
-                        if (s_e[p] < best) {
-                            best = s_e[p];
-                            key = (int)(s_pair[p] & 255);
-                        }
-                }
-                __syncwarp();
-            } else if (np) {  // (rare) too many pairs for the scratch: each row on its own lane
-                const float *xr = sv + lane * d;
-                float best = km_exact(xr, sh.cen + key * kKmMaxD, d);
-                for (unsigned b = cm & (cm - 1); b; b &= b - 1) {
+            }
+            const float nrm = tmem_ld1(tN + t_lane + (uint32_t)sa);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) km_arrive(&B.slotfree[sa]);
+            float m1 = fminf(dd[0], dd[1]);
+#pragma unroll
+            for (int c = 2; c + 1 < NC; c += 2) m1 = fmin3(m1, dd[c], dd[c + 1]);
+            const float thr = m1 + 2.f * 0x1p-14f * (nrm * 1.001f + cmax2);
+            unsigned mask = 0;
+#pragma unroll
+            for (int c = 0; c < NC; ++c) mask |= (dd[c] <= thr ? 1u : 0u) << c;
+            int key = __ffs(mask) - 1;
+            if ((mask & (mask - 1)) && valid) {  // several candidates: E in R18's exact f32 order
+                const float *xgl = pts + (r0 + r) * d;
+                float best = km_exact(xgl, cen_s + key * kKmMaxD, d);
+                for (unsigned b = mask & (mask - 1); b; b &= b - 1) {
                     const int cc = __ffs(b) - 1;
-                    const float e = km_exact(xr, sh.cen + cc * kKmMaxD, d);
-                    if (e < best) {
+                    const float e = km_exact(xgl, cen_s + cc * kKmMaxD, d);
+                    if (e < best) {  // strict <: the first centre wins ties
                         best = e;
                         key = cc;
                     }
                 }
             }
-        }
-        if (lane < kKmRS) {
-            if (lane >= nv) key = kKmK;  // padding row of the partial stage: trash row
-            sk[lane] = key;
-            if (lane < nv) {
-                if (membership) membership[r0 + lane] = key;
-                if (prev) wdelta += (unsigned)(__ldg(prev + r0 + lane) != key);
+            if (valid) {
+                if (membership) membership[r0 + r] = key;
+                wdelta += (unsigned)(prev && pv != key);
             }
-        }
-        __syncwarp();
-        // ---- stream_red accumulation of the stage (as stream_red_tma_s_kernel)
-        int kr[kKmRS];
+            // one-hot B operand of MMA2 (K-major bf16: [centre group][row chunk][8 x 16 B]); the
+            // slot's previous MMA2 is complete (the convert of this stage waited for it)
+            unsigned short *ohs = reinterpret_cast<unsigned short *>(oh + sx * oh_bytes);
+            int op = -1;
 #pragma unroll
-        for (int q = 0; q < kKmRS / 4; ++q) {
-            const int4 v4 = reinterpret_cast<const int4 *>(sk)[q];
-            kr[4 * q] = v4.x;
-            kr[4 * q + 1] = v4.y;
-            kr[4 * q + 2] = v4.z;
-            kr[4 * q + 3] = v4.w;
-        }
-        unsigned B = 0;
+            for (int q = 0; q < kKmNXMax; ++q)
+                if (q == sx) op = ohpos[q];
+            if (op >= 0) ohs[op] = 0;
+            op = valid ? ((key >> 3) * 2048 + (r >> 3) * 128 + (key & 7) * 16 + (r & 7) * 2) / 2 : -1;
+            if (valid) ohs[op] = 0x3F80;  // bf16 1.0
 #pragma unroll
-        for (int r = 0; r < kKmRS; ++r)
-            if (kr[r] == lane) B |= 1u << r;
-        wcnt += (unsigned)__popc(B);
-        float v[kKmRS];
-#pragma unroll
-        for (int r = 0; r < kKmRS; ++r) v[r] = lane < d ? sv[r * d + lane] : 0.f;
-#pragma unroll
-        for (int r = 0; r < kKmRS; ++r) {
-            float *p = s_acc + kr[r] * 32 + lane;
-            *p = __fadd_rn(*p, v[r]);
-        }
-        if (XR > 0)
-            for (unsigned b = B; b; b &= b - 1) {
-                const float *xp = sv + (__ffs(b) - 1) * d + 32;
-#pragma unroll
-                for (int e = 0; e < (XR > 0 ? XR : 1); ++e)
-                    if (e < XW) xa[e] = __fadd_rn(xa[e], xp[e]);
-            }
-        __syncwarp();
-        if (full && lane == 0 && c + kKmStages < nfull) {
+            for (int q = 0; q < kKmNXMax; ++q)
+                if (q == sx) ohpos[q] = op;
             fence_proxy_async();
-            mbar_expect_tx(bars + s, vbytes);
-            tma_load_1d(ring + s * slot, pts + (r0 + (int64_t)kKmStages * kKmRS) * d, vbytes, bars + s);
+            __syncwarp();
+            if (lane == 0) km_arrive(&B.ohfull[sx]);
+            if (flushed < nseg2 && (flushed + 1) * kKmSeg + 1 <= s) flush();
         }
-        if (full && ++s == kKmStages) {
-            s = 0;
-            phase ^= 1u;
+        while (flushed < nseg2) flush();
+        wdelta = __reduce_add_sync(0xffffffffu, wdelta);
+        if (lane == 0 && wdelta) atomicAdd(gdelta, (unsigned long long)wdelta);
+        // every MMA has completed (the last D2 buffer follows every MMA2): the X slots may hold
+        // the partial
+        km_bar_sync(1, 4 * 32);
+#pragma unroll
+        for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c];
+    } else if (warp == kKmWarpProd) {
+        // =============================== producer: TMA bulk copies of full stages
+        if (lane == 0) {
+            for (int s = 0; s < nfull; ++s) {
+                const int slot = s % NR;
+                if (s >= NR) km_wait(&B.raw_empty[slot], (unsigned)(((s / NR) - 1) & 1));
+                mbar_expect_tx(&B.raw_full[slot], raw_bytes);
+                km_tma_load(raw + slot * raw_slot, pts + (i0 + (int64_t)s * kKmRows) * d, raw_bytes,
+                            &B.raw_full[slot]);
+            }
+        }
+    } else {
+        // =============================== MMA issuer (one thread)
+        if (lane == 0) {
+            constexpr uint32_t id1 = umma_idesc_bf16(N1, 0, 0);
+            constexpr uint32_t id2 = umma_idesc_bf16(NC, 1, 0);  // A (X) MN-major, B (one-hot) K-major
+            const uint32_t x20 = km_smem(x2), oh0 = km_smem(oh), b10 = km_smem(b1);
+            const int K1S = 2 * G.KP / 16;  // MMA1 instructions (K = 16 each)
+            int s1 = 0, s2 = 0;
+            while (s2 < ns) {
+                if (s1 < ns && km_test(&B.a1full[s1 % kKmNA], (unsigned)((s1 / kKmNA) & 1))) {
+                    tc_fence_after();
+                    const int sa = s1 % kKmNA;
+                    const uint32_t ta = tA + (uint32_t)(sa * G.KP), dt = tD1 + (uint32_t)(sa * N1);
+                    for (int p = 0; p < K1S; ++p)  // 8 TMEM columns (16 bf16) of A per instruction
+                        umma_bf16_ts(dt, ta + 8 * p, umma_desc(b10 + p * 256, 128, SB1), id1, p > 0);
+                    umma_commit(&B.d1full[sa]);
+                    ++s1;
+                }
+                if (s2 < s1 && km_test(&B.ohfull[s2 % NX], (unsigned)((s2 / NX) & 1))) {
+                    const int seg = s2 / kKmSeg, b2 = seg & 1;
+                    const bool first = (s2 % kKmSeg) == 0;
+                    if (!first || seg < 2 || km_test(&B.d2free[b2], (unsigned)(((seg >> 1) - 1) & 1))) {
+                        tc_fence_after();
+                        const int sx = s2 % NX;
+                        const uint32_t xa = x20 + sx * x2_bytes, ob = oh0 + sx * oh_bytes;
+                        const uint32_t dt = tD2 + (uint32_t)(b2 * NC);
+#pragma unroll 4
+                        for (int kk = 0; kk < kKmRows / 16; ++kk)  // K = 16 rows per instruction
+                            umma_bf16_ss(dt, umma_desc(xa + kk * 2 * LB2, LB2, 128), umma_desc(ob + kk * 256, 128, 2048),
+                                         id2, (first && kk == 0) ? 0u : 1u);
+                        umma_commit(&B.x2free[sx]);
+                        if ((s2 + 1) % kKmSeg == 0 || s2 + 1 == ns) umma_commit(&B.d2full[b2]);
+                        ++s2;
+                    }
+                }
+            }
         }
     }
-    // ---- chunk results -> CTA (warp order) -> workspace; last CTA -> outputs
-    wdelta = __reduce_add_sync(0xffffffffu, wdelta);
-    if (lane == 0 && wdelta) atomicAdd(gdelta, (unsigned long long)wdelta);
+    tc_fence_before();
     __syncthreads();
-    float *s_kw = reinterpret_cast<float *>(smem);  // [k][d] CTA sums (reuses warp 0's ring)
-    int *s_cnt = reinterpret_cast<int *>(smem + align_up((size_t)kKmK * kKmMaxD * 4, 16));
-    // each warp's region is still intact except warp 0's ring: combine through registers
-    float colsum[kKmK];  // lane j: column j of every cluster, summed over warps in order
-#pragma unroll
-    for (int cc = 0; cc < kKmK; ++cc) colsum[cc] = 0.f;
-    __syncthreads();
-    if (warp == 0) {
-        for (int q = 0; q < kKmWarps; ++q) {
-            const float *qa = reinterpret_cast<const float *>(smem + (size_t)q * warp_bytes + kKmStages * slot +
-                                                              kKmStages * 8);
-#pragma unroll
-            for (int cc = 0; cc < kKmK; ++cc) colsum[cc] = __fadd_rn(colsum[cc], qa[cc * 32 + lane]);
-        }
+    if (warp == kKmWarpMma) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
     }
-    __syncthreads();  // warp 0 has read every accumulator; the rings may now be reused
-    // extras and counts: per-warp values held by the cluster-owner lanes -> shared, warp order
-    float *s_x = reinterpret_cast<float *>(smem + align_up((size_t)kKmK * kKmMaxD * 4, 16) + 256);  // [W][K][XR]
-    int *s_wc = reinterpret_cast<int *>(smem + align_up((size_t)kKmK * kKmMaxD * 4, 16) + 256 +
-                                        (size_t)kKmWarps * kKmK * kKmXR * 4);  // [W][K]
-#pragma unroll
-    for (int e = 0; e < kKmXR; ++e) s_x[(warp * kKmK + lane) * kKmXR + e] = e < XR ? xa[e < XR ? e : 0] : 0.f;
-    s_wc[warp * kKmK + lane] = (int)wcnt;
-    if (warp == 0 && lane < d) {
-#pragma unroll
-        for (int cc = 0; cc < kKmK; ++cc)
-            if (cc < k) s_kw[cc * d + lane] = colsum[cc];
-    }
-    __syncthreads();
-    for (int e = threadIdx.x; e < k * d; e += kKmThreads) {
-        const int cc = e / d, j = e - cc * d;
-        if (j >= 32) {
-            float a = 0.f;
-            for (int q = 0; q < kKmWarps; ++q) a = __fadd_rn(a, s_x[(q * kKmK + cc) * kKmXR + (j - 32)]);
-            s_kw[e] = a;
-        }
-    }
-    if (threadIdx.x < k) {
-        unsigned a = 0;
-        for (int q = 0; q < kKmWarps; ++q) a += (unsigned)s_wc[q * kKmK + threadIdx.x];
-        s_cnt[threadIdx.x] = (int)a;
-    }
-    __syncthreads();
+    // ---- CTA partial: sums[c][j] = a1 row j + a2 row JB + j; counts = row d
     const int64_t kd = (int64_t)k * d;
-    for (int64_t e = threadIdx.x; e < kd; e += kKmThreads) __stcg(partials + blockIdx.x * kd + e, s_kw[e]);
-    for (int cc = threadIdx.x; cc < k; cc += kKmThreads) __stcg(pcounts + blockIdx.x * k + cc, s_cnt[cc]);
+    for (int64_t e = tid; e < kd; e += kKmThreads) {
+        const int c = (int)(e / d), j = (int)(e - (int64_t)c * d);
+        __stcg(partials + blockIdx.x * kd + e, __fadd_rn(s_part[j * NC + c], s_part[(G.JB + j) * NC + c]));
+    }
+    for (int c = tid; c < k; c += kKmThreads) __stcg(pcounts + blockIdx.x * k + c, (int)s_part[d * NC + c]);
     __shared__ bool last;
+    __shared__ int s_cnt[kKmK];
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
         __threadfence();
         last = atomicAdd(ticket, 1u) == gridDim.x - 1;
         if (last) __threadfence();
     }
     __syncthreads();
     if (!last) return;
-    const int G = gridDim.x;
+    const int NCTA = gridDim.x;
     // four interleaved accumulators (a fixed order): ~32 independent L2 loads in flight
-    for (int cc = threadIdx.x; cc < k; cc += kKmThreads) {
+    for (int cc = tid; cc < k; cc += kKmThreads) {
         unsigned a0 = 0, a1 = 0, a2 = 0, a3 = 0;
         int q = 0;
 #pragma unroll 8
-        for (; q + 4 <= G; q += 4) {
+        for (; q + 4 <= NCTA; q += 4) {
             const int *p = pcounts + (int64_t)q * k + cc;
             a0 += (unsigned)__ldcg(p);
             a1 += (unsigned)__ldcg(p + k);
             a2 += (unsigned)__ldcg(p + 2 * k);
             a3 += (unsigned)__ldcg(p + 3 * k);
         }
-        for (; q < G; ++q) a0 += (unsigned)__ldcg(pcounts + (int64_t)q * k + cc);
+        for (; q < NCTA; ++q) a0 += (unsigned)__ldcg(pcounts + (int64_t)q * k + cc);
         const unsigned a = a0 + a1 + a2 + a3;
         s_cnt[cc] = (int)a;
         counts[cc] = (int32_t)a;
     }
     __syncthreads();
-    for (int64_t e = threadIdx.x; e < kd; e += kKmThreads) {
+    for (int64_t e = tid; e < kd; e += kKmThreads) {
         float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
         int q = 0;
 #pragma unroll 8
-        for (; q + 4 <= G; q += 4) {
+        for (; q + 4 <= NCTA; q += 4) {
             const float *p = partials + (int64_t)q * kd + e;
             a0 = __fadd_rn(a0, __ldcg(p));
             a1 = __fadd_rn(a1, __ldcg(p + kd));
             a2 = __fadd_rn(a2, __ldcg(p + 2 * kd));
             a3 = __fadd_rn(a3, __ldcg(p + 3 * kd));
         }
-        for (; q < G; ++q) a0 = __fadd_rn(a0, __ldcg(partials + (int64_t)q * kd + e));
+        for (; q < NCTA; ++q) a0 = __fadd_rn(a0, __ldcg(partials + (int64_t)q * kd + e));
         const float a = __fadd_rn(__fadd_rn(a0, a1), __fadd_rn(a2, a3));
         sums[e] = a;
         const int cc = (int)(e / d);
         if (new_cen) new_cen[e] = s_cnt[cc] > 0 ? __fdiv_rn(a, (float)s_cnt[cc]) : cen[e];
     }
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
         if (delta_out) *delta_out = prev ? (int64_t)__ldcg(gdelta) : 0;
         *gdelta = 0;
         atomicExch(ticket, 0u);
     }
 }
 
-static size_t km_warp_bytes(int64_t d) {
-    return (size_t)kKmStages * ((size_t)kKmRS * d * 4 + kKmRS * 4) + kKmStages * 8 + (size_t)(kKmK + 1) * 32 * 4 +
-           kKmPairs * 8;
+static size_t km_smem_bytes(int64_t d, int NC, int NR, int NX) {
+    const KmGeom G((int)d);
+    const size_t raw_slot = align_up((size_t)kKmRows * d * 4, 1024);
+    const size_t oh = (size_t)NC / 8 * 2048;
+    const size_t b1 = (size_t)(2 * NC / 8) * (2 * G.KP / 8 * 128);
+    return 1024 + NR * raw_slot + NX * ((size_t)G.x2_bytes() + oh) + 1024 + b1 + (size_t)NC * kKmMaxD * 4 +
+           sizeof(KmBars);
 }
-static size_t km_smem(int64_t d) {
-    const size_t a = (size_t)kKmWarps * km_warp_bytes(d) + sizeof(KmShared);
-    // combine scratch (carved from the start of the rings): sums, counts, extras, per-warp counts
-    const size_t b = align_up((size_t)kKmK * kKmMaxD * 4, 16) + 256 + (size_t)kKmWarps * kKmK * kKmXR * 4 +
-                     (size_t)kKmWarps * kKmK * 4;
-    return a > b ? a : b;
+// deepest rings that fit the 227 KB opt-in limit (+ the static shared words): X slots first
+static void km_rings(int64_t d, int NC, int &NR, int &NX) {
+    for (NX = kKmNXMax; NX >= 2; --NX)
+        for (NR = kKmRing; NR >= 3; --NR)
+            if (km_smem_bytes(d, NC, NR, NX) + 2048 <= 227 * 1024) return;
+    NR = 2;
+    NX = 2;
 }
 static int64_t km_grid(int64_t n) {
-    int64_t warps = ceil_div(n, 4 * kKmRS);  // at least 4 stages per warp
-    const int64_t cap = (int64_t)sm_count() * 2 * kKmWarps;
-    if (warps > cap) warps = cap;
-    if (warps < 1) warps = 1;
-    return ceil_div(warps, kKmWarps);
+    const int64_t stages = ceil_div(n, kKmRows);
+    int64_t g = sm_count();
+    if (stages < g) g = stages;
+    return g < 1 ? 1 : g;
 }
 
 size_t kmeans_ws(int64_t n, int64_t d, int64_t k) {
-    const int64_t G = (int64_t)sm_count() * 2;  // >= km_grid(n)
+    const int64_t G = (int64_t)sm_count();  // >= km_grid(n)
     (void)n;
     return kWsHeader + align_up((size_t)G * k * d * 4, 256) + align_up((size_t)G * k * 4, 256);
 }
 
-template <int KS, int XR>
+template <int NC, int DT>
 static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen, int k, const int32_t *prev,
                            int32_t *membership, float *sums, int32_t *counts, float *new_cen, int64_t *delta,
                            void *ws, cudaStream_t st) {
     const int64_t G = km_grid(n);
-    const int64_t warps = G * kKmWarps;
-    int64_t rows = n > 0 ? ceil_div(n, warps) : 0;
-    rows = ceil_div(rows, kKmRS) * kKmRS;  // stages start 16-row (64d-byte) aligned
+    const int64_t rows = ceil_div(ceil_div(n > 0 ? n : 1, G), kKmRows) * kKmRows;  // whole stages per CTA
     char *w = (char *)ws;
     unsigned long long *gdelta = (unsigned long long *)(w + kWsCount2);  // zero between calls (header)
     float *parts = (float *)(w + kWsHeader);
     int *pcnt = (int *)(w + kWsHeader + align_up((size_t)G * k * d * 4, 256));
-    const size_t smem = km_smem(d);
-    cudaFuncSetAttribute((const void *)kmeans_step_kernel<KS, XR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)smem);
-    kmeans_step_kernel<KS, XR><<<(unsigned)G, kKmThreads, smem, st>>>(pts, n, d, cen, k, prev, membership, rows, parts,
-                                                                   pcnt, (unsigned *)(w + kWsTicket), gdelta, sums,
-                                                                   counts, new_cen, delta);
+    int NR, NX;
+    km_rings(d, NC, NR, NX);
+    const size_t smem = km_smem_bytes(d, NC, NR, NX);
+    auto kern = kmeans_tc_kernel<NC, DT>;
+    cudaFuncSetAttribute((const void *)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    kern<<<(unsigned)G, kKmThreads, smem, st>>>(pts, n, d, NR, NX, cen, k, prev, membership, rows, parts, pcnt,
+                                                 (unsigned *)(w + kWsTicket), gdelta, sums, counts, new_cen, delta);
     return launch_status();
 }
 
 fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, int64_t k, const int32_t *prev,
                      int32_t *membership, float *sums, int32_t *counts, float *new_cen, int64_t *delta, void *ws,
                      cudaStream_t st) {
-#define FS_KM(KS, XR) return km_launch<KS, XR>(pts, n, (int)d, cen, (int)k, prev, membership, sums, counts, new_cen, delta, ws, st)
-    if (d <= 8) FS_KM(1, 0);
-    if (d <= 16) FS_KM(2, 0);
-    if (d <= 24) FS_KM(3, 0);
-    if (d <= 32) FS_KM(4, 0);
-    if (d <= 34) FS_KM(5, 2);
-    if (d <= 36) FS_KM(5, 4);
-    if (d <= 40) FS_KM(5, 8);
-#undef FS_KM
-    return FS_ERR_UNSUPPORTED;
+    // d = 34 (the kdd_cup width of C3 / C5) is compiled with the width known; others at run time
+    if (k <= 16)
+        return d == 34 ? km_launch<16, 34>(pts, n, (int)d, cen, (int)k, prev, membership, sums, counts, new_cen, delta,
+                                           ws, st)
+                       : km_launch<16, 0>(pts, n, (int)d, cen, (int)k, prev, membership, sums, counts, new_cen, delta,
+                                          ws, st);
+    return d == 34 ? km_launch<32, 34>(pts, n, (int)d, cen, (int)k, prev, membership, sums, counts, new_cen, delta, ws,
+                                       st)
+                   : km_launch<32, 0>(pts, n, (int)d, cen, (int)k, prev, membership, sums, counts, new_cen, delta, ws,
+                                      st);
 }
 
 // new centres from (already combined) sums and counts: the last step of the iteration
