@@ -49,10 +49,13 @@ namespace fs {
 constexpr int kKmRows = 128;   // rows per stage (UMMA M)
 constexpr int kKmRing = 5;     // TMA ring slots (at most)
 constexpr int kKmCv = 2;       // convert groups of 4 warps; group g converts stages s = g (mod 2)
-constexpr int kKmNA = 3;       // TMEM stage slots (A operand, |x|^2, D1)
-constexpr int kKmNXMax = 4;    // shared-memory stage slots (MMA2 operands), at most
-constexpr int kKmThreads = (4 * kKmCv + 4 + 2) * 32;  // convert + decide + producer + MMA warp
-constexpr int kKmWarpDecide = 4 * kKmCv, kKmWarpProd = 4 * kKmCv + 4, kKmWarpMma = 4 * kKmCv + 5;
+constexpr int kKmNA = 4;       // TMEM stage slots (A operand, D1)
+constexpr int kKmDc = 2;       // decide groups of 4 warps; group g decides stages s = g (mod 2)
+constexpr int kKmNXMax = 6;    // shared-memory stage slots (MMA2 operands), at most
+constexpr int kKmThreads = (4 * kKmCv + 4 * kKmDc + 3) * 32;  // convert + decide + producer + 2 MMA warps
+constexpr int kKmWarpDecide = 4 * kKmCv, kKmWarpProd = 4 * (kKmCv + kKmDc), kKmWarpMma = kKmWarpProd + 1;
+// (MMA1 and MMA2 are issued by two warps, kKmWarpMma and kKmWarpMma + 1: a tcgen05.mma occupies
+// its issuing thread for ~100+ cycles, one issuer alone could not keep up with both streams)
 constexpr int kKmK = 32;       // max clusters
 constexpr int kKmMaxD = 40;
 constexpr int kKmSeg = 16;     // stages per D2 buffer
@@ -184,6 +187,16 @@ __device__ __forceinline__ float km_exact(const float *x, const float *c, int d)
 
 
 
+// Debug tracing (tools/km_trace.py): clock64 stamps of CTA 0's pipeline events per stage when
+// FUTSEG_KM_TRACE is set; [stage][8]: convert begin / ready / end, decide begin / ready / end,
+// MMA1 issue, MMA2 issue.
+__device__ long long *g_km_trace = nullptr;
+
+#define KM_TRACE(s, e)                                                                   \
+    do {                                                                                 \
+        if (trace && (threadIdx.x & 127) == 0) trace[(s) * 16 + (e)] = clock64();         \
+    } while (0)
+
 struct KmBars {
     uint64_t raw_full[kKmRing], raw_empty[kKmRing];
     uint64_t a1full[kKmNA], d1full[kKmNA], slotfree[kKmNA];
@@ -191,7 +204,9 @@ struct KmBars {
     uint64_t d2full[2], d2free[2];
     uint32_t tmem_base;
     float cmax2;
+    float nrm[kKmNA][kKmRows];  // |x|^2 of the rows of the stages in the TMEM slots
 };
+// running f32 totals of the D2 buffers ([128 M rows][NC]), after the barriers in shared memory
 
 // Operand geometry for a given d (host and device):
 //   KP  = bf16 columns of one A piece: d + 3 augmentation columns, padded to 16
@@ -211,13 +226,15 @@ __device__ __forceinline__ uint32_t cvt_bf2(float lo, float hi) {  // packed bf1
     return r;
 }
 
+__device__ int g_km_skip = 0;  // debug: bit 0 skips the MMA2 instructions, bit 1 the MMA1 ones, bit 2 the
+                               // A stores to TMEM, bit 3 the X stores to shared memory (timing only)
 // One row of a stage -> the two bf16 pieces of every column, written as the MMA1 A operand (TMEM
 // lane of the calling thread, K-major pairs: [a1 | 1 1 1 | 0..] then [a2 | 0..], KP columns each)
 // and as the MMA2 A operand (shared memory, MN-major: the row is the K index, a1 rows 0..d-1, the
 // count row d, a2 rows JB..JB+d-1).  Returns |x|^2 (f32).
 template <bool FULL, bool EVEN>
 __device__ __forceinline__ float km_convert_row(const float *src, int d, bool valid, const KmGeom &G, int qd,
-                                                uint32_t ta, unsigned char *xr) {
+                                                uint32_t ta, unsigned char *xr, int skip) {
     float nrm = 0.f;
 #pragma unroll
     for (int q = 0; q < 3; ++q) {  // 16 columns per chunk (KP <= 48)
@@ -260,8 +277,11 @@ __device__ __forceinline__ float km_convert_row(const float *src, int d, bool va
                     wx[t] |= ((j0 == d && valid) ? 0x3F80u : 0u) | ((j1 == d && valid) ? 0x3F800000u : 0u);
                 }
             }
-            tmem_st8u(ta + 8 * q, wt);
-            tmem_st8u(ta + G.KP / 2 + 8 * q, w2);
+            if (!(skip & 4)) {
+                tmem_st8u(ta + 8 * q, wt);
+                tmem_st8u(ta + G.KP / 2 + 8 * q, w2);
+            }
+            if (skip & 8) continue;
             if (16 * q < G.JB) *reinterpret_cast<uint4 *>(xr + (2 * q) * 128) = make_uint4(wx[0], wx[1], wx[2], wx[3]);
             if (16 * q + 8 < G.JB)
                 *reinterpret_cast<uint4 *>(xr + (2 * q + 1) * 128) = make_uint4(wx[4], wx[5], wx[6], wx[7]);
@@ -285,6 +305,8 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int d = DT > 0 ? DT : d_rt;  // DT > 0: the width is a compile-time constant (C3 / C5: 34)
+    long long *const trace = blockIdx.x == 0 ? g_km_trace : nullptr;  // debug tracing (normally null)
+    const int skip = g_km_skip;                                        // debug timing switches (0)
     constexpr bool EVEN = DT > 0 && DT % 2 == 0;
     const KmGeom G(d);
     constexpr int N1 = 2 * NC;  // MMA1 N: (centre, b piece)
@@ -301,6 +323,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     unsigned char *b1 = oh + NX * oh_bytes;                 // [N1/8][K1/8][8 x 16 B]
     float *cen_s = reinterpret_cast<float *>(b1 + (N1 / 8) * SB1);  // [NC][kKmMaxD]
     KmBars &B = *reinterpret_cast<KmBars *>(cen_s + NC * kKmMaxD);
+    float *s_acc = reinterpret_cast<float *>(&B + 1);  // [128][NC]
 
     const int64_t i0 = (int64_t)blockIdx.x * rows_per_cta;
     const int64_t i1 = i0 + rows_per_cta < n ? i0 + rows_per_cta : n;
@@ -383,8 +406,8 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = B.tmem_base;
-    // TMEM columns: D1 slots [0, NA N1), D2 buffers (2 NC), |x|^2 (32), A slots (KP each)
-    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tN = tD2 + 2 * NC, tA = tN + 32;
+    // TMEM columns: D1 slots [0, NA N1), D2 buffers (2 NC), A slots (KP each): <= 4 64 + 64 + 4 48 = 512
+    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tA = tD2 + 2 * NC;
 
     float *s_part = reinterpret_cast<float *>(x2);  // [128][NC] CTA partial (after the loop)
     if (warp < kKmWarpDecide) {
@@ -399,6 +422,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             const int nv = full ? kKmRows : (int)(i1 - r0);
             const bool valid = r < nv;
             const float *src;
+            KM_TRACE(s, 0);
             if (full) {
                 km_wait(&B.raw_full[s % NR], (unsigned)((s / NR) & 1));
                 src = reinterpret_cast<const float *>(raw + (s % NR) * raw_slot) + (size_t)r * d;
@@ -411,12 +435,13 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             tc_fence_after();
             const uint32_t ta = tA + t_lane + (uint32_t)(sa * G.KP);
             unsigned char *xr = x2 + sx * x2_bytes + (r >> 3) * LB2 + (r & 7) * 16;
+            KM_TRACE(s, 1);
             float nrm;
             if (full)
-                nrm = km_convert_row<true, EVEN>(src, d, true, G, qd, ta, xr);
+                nrm = km_convert_row<true, EVEN>(src, d, true, G, qd, ta, xr, skip);
             else
-                nrm = km_convert_row<false, EVEN>(src, d, valid, G, qd, ta, xr);
-            tmem_st1(tN + t_lane + (uint32_t)sa, nrm);
+                nrm = km_convert_row<false, EVEN>(src, d, valid, G, qd, ta, xr, skip);
+            B.nrm[sa][r] = nrm;
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
             fence_proxy_async();
             tc_fence_before();
@@ -425,16 +450,17 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
                 if (full) km_arrive(&B.raw_empty[s % NR]);
                 km_arrive(&B.a1full[sa]);
             }
+            KM_TRACE(s, 2);
         }
     } else if (warp < kKmWarpProd) {
         // =============================== decide: candidates from the tensor-core ranking, exact R18
         // for near-ties; one-hot MMA2 operand; membership; delta; D2 buffers -> registers
-        const int wl = warp - kKmWarpDecide, r = wl * 32 + lane;
+        const int dg = (warp - kKmWarpDecide) >> 2, wl = warp & 3, r = wl * 32 + lane;
         const uint32_t t_lane = (uint32_t)(wl * 32) << 16;
         const float cmax2 = B.cmax2;
-        float acc_tot[NC];
-#pragma unroll
-        for (int c = 0; c < NC; ++c) acc_tot[c] = 0.f;
+        float *acc_tot = s_acc + r * NC;  // this thread's M row of the D2 totals (group 0)
+        if (dg == 0)
+            for (int c = 0; c < NC; ++c) acc_tot[c] = 0.f;
         int ohpos[kKmNXMax];
 #pragma unroll
         for (int q = 0; q < kKmNXMax; ++q) ohpos[q] = -1;
@@ -453,13 +479,15 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             if (lane == 0) km_arrive(&B.d2free[b2]);
             ++flushed;
         };
-        for (int s = 0; s < ns; ++s) {
+        for (int s = dg; s < ns; s += kKmDc) {
             const int64_t r0 = i0 + (int64_t)s * kKmRows;
             const int nv = s < nfull ? kKmRows : (int)(i1 - r0);
             const bool valid = r < nv;
             const int sa = s % kKmNA, sx = s % NX;
             const int pv = (prev && valid) ? __ldg(prev + r0 + r) : 0;  // in flight during the wait
+            KM_TRACE(s, 3);
             km_wait(&B.d1full[sa], (unsigned)((s / kKmNA) & 1));
+            km_wait(&B.a1full[sa], (unsigned)((s / kKmNA) & 1));  // (complete: orders the |x|^2 store)
             tc_fence_after();
             float dd[NC];
             {
@@ -476,7 +504,8 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
                     for (int c = 0; c < NC; ++c) dd[c] = __fadd_rn(dd[c], v[NC + c]);
                 }
             }
-            const float nrm = tmem_ld1(tN + t_lane + (uint32_t)sa);
+            const float nrm = B.nrm[sa][r];
+            KM_TRACE(s, 4);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) km_arrive(&B.slotfree[sa]);
@@ -486,7 +515,11 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             const float thr = m1 + 2.f * 0x1p-14f * (nrm * 1.001f + cmax2);
             unsigned mask = 0;
 #pragma unroll
-            for (int c = 0; c < NC; ++c) mask |= (dd[c] <= thr ? 1u : 0u) << c;
+            for (int c = 0; c < NC; ++c) {
+                uint32_t le;
+                asm("set.le.u32.f32 %0, %1, %2;" : "=r"(le) : "f"(dd[c]), "f"(thr));
+                mask |= le & (1u << c);
+            }
             int key = __ffs(mask) - 1;
             if ((mask & (mask - 1)) && valid) {  // several candidates: E in R18's exact f32 order
                 const float *xgl = pts + (r0 + r) * d;
@@ -520,16 +553,18 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             fence_proxy_async();
             __syncwarp();
             if (lane == 0) km_arrive(&B.ohfull[sx]);
-            if (flushed < nseg2 && (flushed + 1) * kKmSeg + 1 <= s) flush();
+            KM_TRACE(s, 5);
+            if (dg == 0 && flushed < nseg2 && (flushed + 1) * kKmSeg + 1 <= s) flush();  // group 0 owns D2
         }
-        while (flushed < nseg2) flush();
+        if (dg == 0)
+            while (flushed < nseg2) flush();
         wdelta = __reduce_add_sync(0xffffffffu, wdelta);
         if (lane == 0 && wdelta) atomicAdd(gdelta, (unsigned long long)wdelta);
         // every MMA has completed (the last D2 buffer follows every MMA2): the X slots may hold
         // the partial
-        km_bar_sync(1, 4 * 32);
-#pragma unroll
-        for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c];
+        km_bar_sync(1, 4 * kKmDc * 32);
+        if (dg == 0)
+            for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c];
     } else if (warp == kKmWarpProd) {
         // =============================== producer: TMA bulk copies of full stages
         if (lane == 0) {
@@ -542,40 +577,46 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             }
         }
     } else {
-        // =============================== MMA issuer (one thread)
-        if (lane == 0) {
-            constexpr uint32_t id1 = umma_idesc_bf16(N1, 0, 0);
-            constexpr uint32_t id2 = umma_idesc_bf16(NC, 1, 0);  // A (X) MN-major, B (one-hot) K-major
-            const uint32_t x20 = km_smem(x2), oh0 = km_smem(oh), b10 = km_smem(b1);
+        // =============================== MMA issuers: one thread for MMA1, one for MMA2
+        constexpr uint32_t id1 = umma_idesc_bf16(N1, 0, 0);
+        constexpr uint32_t id2 = umma_idesc_bf16(NC, 1, 0);  // A (X) MN-major, B (one-hot) K-major
+        if (warp == kKmWarpMma && lane == 0) {
+            const uint32_t b10 = km_smem(b1);
             const int K1S = 2 * G.KP / 16;  // MMA1 instructions (K = 16 each)
-            int s1 = 0, s2 = 0;
-            while (s2 < ns) {
-                if (s1 < ns && km_test(&B.a1full[s1 % kKmNA], (unsigned)((s1 / kKmNA) & 1))) {
-                    tc_fence_after();
-                    const int sa = s1 % kKmNA;
-                    const uint32_t ta = tA + (uint32_t)(sa * G.KP), dt = tD1 + (uint32_t)(sa * N1);
-                    for (int p = 0; p < K1S; ++p)  // 8 TMEM columns (16 bf16) of A per instruction
-                        umma_bf16_ts(dt, ta + 8 * p, umma_desc(b10 + p * 256, 128, SB1), id1, p > 0);
-                    umma_commit(&B.d1full[sa]);
-                    ++s1;
-                }
-                if (s2 < s1 && km_test(&B.ohfull[s2 % NX], (unsigned)((s2 / NX) & 1))) {
-                    const int seg = s2 / kKmSeg, b2 = seg & 1;
-                    const bool first = (s2 % kKmSeg) == 0;
-                    if (!first || seg < 2 || km_test(&B.d2free[b2], (unsigned)(((seg >> 1) - 1) & 1))) {
-                        tc_fence_after();
-                        const int sx = s2 % NX;
-                        const uint32_t xa = x20 + sx * x2_bytes, ob = oh0 + sx * oh_bytes;
-                        const uint32_t dt = tD2 + (uint32_t)(b2 * NC);
-#pragma unroll 4
-                        for (int kk = 0; kk < kKmRows / 16; ++kk)  // K = 16 rows per instruction
-                            umma_bf16_ss(dt, umma_desc(xa + kk * 2 * LB2, LB2, 128), umma_desc(ob + kk * 256, 128, 2048),
-                                         id2, (first && kk == 0) ? 0u : 1u);
-                        umma_commit(&B.x2free[sx]);
-                        if ((s2 + 1) % kKmSeg == 0 || s2 + 1 == ns) umma_commit(&B.d2full[b2]);
-                        ++s2;
-                    }
-                }
+            const uint64_t bdesc0 = umma_desc(b10, 128, SB1);
+            for (int s1 = 0; s1 < ns; ++s1) {
+                const int sa = s1 % kKmNA;
+                km_wait(&B.a1full[sa], (unsigned)((s1 / kKmNA) & 1));  // (implies the D1 slot is free)
+                if (trace) trace[s1 * 16 + 8] = clock64();
+                tc_fence_after();
+                const uint32_t ta = tA + (uint32_t)(sa * G.KP), dt = tD1 + (uint32_t)(sa * N1);
+                for (int p = 0; p < ((skip & 2) ? 0 : K1S); ++p)  // 8 TMEM columns (16 bf16) of A each
+                    umma_bf16_ts(dt, ta + 8 * p, bdesc0 + (uint64_t)(p * 256 >> 4), id1, p > 0);
+                if (trace) trace[s1 * 16 + 9] = clock64();
+                umma_commit(&B.d1full[sa]);
+                if (trace) trace[s1 * 16 + 6] = clock64();
+            }
+        } else if (warp == kKmWarpMma + 1 && lane == 0) {
+            const uint32_t x20 = km_smem(x2), oh0 = km_smem(oh);
+            for (int s2 = 0; s2 < ns; ++s2) {
+                const int sx = s2 % NX, seg = s2 / kKmSeg, b2 = seg & 1;
+                const bool first = (s2 % kKmSeg) == 0;
+                km_wait(&B.ohfull[sx], (unsigned)((s2 / NX) & 1));  // (implies MMA1 of the stage is done)
+                if (first && seg >= 2) km_wait(&B.d2free[b2], (unsigned)(((seg >> 1) - 1) & 1));
+                if (trace) trace[s2 * 16 + 10] = clock64();
+                tc_fence_after();
+                const uint64_t ad = umma_desc(x20 + sx * x2_bytes, LB2, 128);
+                const uint64_t bd = umma_desc(oh0 + sx * oh_bytes, 128, 2048);
+                const uint32_t dt = tD2 + (uint32_t)(b2 * NC);
+#pragma unroll
+                for (int kk = 0; kk < kKmRows / 16; ++kk)  // K = 16 rows per instruction
+                    if (!(skip & 1))
+                        umma_bf16_ss(dt, ad + (uint64_t)((kk * 2 * LB2) >> 4), bd + (uint64_t)((kk * 256) >> 4), id2,
+                                     (first && kk == 0) ? 0u : 1u);
+                if (trace) trace[s2 * 16 + 11] = clock64();
+                umma_commit(&B.x2free[sx]);
+                if (trace) trace[s2 * 16 + 7] = clock64();
+                if ((s2 + 1) % kKmSeg == 0 || s2 + 1 == ns) umma_commit(&B.d2full[b2]);
             }
         }
     }
@@ -651,11 +692,12 @@ static size_t km_smem_bytes(int64_t d, int NC, int NR, int NX) {
     const size_t oh = (size_t)NC / 8 * 2048;
     const size_t b1 = (size_t)(2 * NC / 8) * (2 * G.KP / 8 * 128);
     return 1024 + NR * raw_slot + NX * ((size_t)G.x2_bytes() + oh) + 1024 + b1 + (size_t)NC * kKmMaxD * 4 +
-           sizeof(KmBars);
+           sizeof(KmBars) + (size_t)kKmRows * NC * 4;
 }
 // deepest rings that fit the 227 KB opt-in limit (+ the static shared words): X slots first
 static void km_rings(int64_t d, int NC, int &NR, int &NX) {
-    for (NX = kKmNXMax; NX >= 2; --NX)
+    // NX even: a slot is always reused by the same decide group (it resets its own one-hot entries)
+    for (NX = kKmNXMax; NX >= 2; NX -= kKmDc)
         for (NR = kKmRing; NR >= 3; --NR)
             if (km_smem_bytes(d, NC, NR, NX) + 2048 <= 227 * 1024) return;
     NR = 2;
@@ -686,12 +728,28 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
     int *pcnt = (int *)(w + kWsHeader + align_up((size_t)G * k * d * 4, 256));
     int NR, NX;
     km_rings(d, NC, NR, NX);
+    {
+        static long long *tr = nullptr;
+        const char *e = getenv("FUTSEG_KM_TRACE");
+        if (e && !tr) cudaMalloc(&tr, 16 * 8 * 8192);
+        long long *p = e ? tr : nullptr;
+        cudaMemcpyToSymbolAsync(g_km_trace, &p, sizeof(p), 0, cudaMemcpyHostToDevice, st);
+        static int skip = getenv("FUTSEG_KM_SKIP") ? atoi(getenv("FUTSEG_KM_SKIP")) : 0;
+        cudaMemcpyToSymbolAsync(g_km_skip, &skip, sizeof(skip), 0, cudaMemcpyHostToDevice, st);
+    }
     const size_t smem = km_smem_bytes(d, NC, NR, NX);
     auto kern = kmeans_tc_kernel<NC, DT>;
     cudaFuncSetAttribute((const void *)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     kern<<<(unsigned)G, kKmThreads, smem, st>>>(pts, n, d, NR, NX, cen, k, prev, membership, rows, parts, pcnt,
                                                  (unsigned *)(w + kWsTicket), gdelta, sums, counts, new_cen, delta);
     return launch_status();
+}
+
+// FUTSEG_KM_TRACE: copy CTA 0's stage stamps to the host (tools/km_trace.py)
+extern "C" int fs_debug_km_trace(long long *host, int nstages) {
+    long long *p = nullptr;
+    if (cudaMemcpyFromSymbol(&p, g_km_trace, sizeof(p)) != cudaSuccess || !p) return 1;
+    return cudaMemcpy(host, p, (size_t)nstages * 16 * 8, cudaMemcpyDeviceToHost) == cudaSuccess ? 0 : 1;
 }
 
 fs_status kmeans_run(const float *pts, int64_t n, int64_t d, const float *cen, int64_t k, const int32_t *prev,

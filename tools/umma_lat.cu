@@ -65,6 +65,29 @@ __global__ void lat(long long *out, int mode, int reps) {
                 const uint32_t idn = (1u << 4) | (2u << 7) | (2u << 10) | ((N >> 3) << 17) | ((128u >> 4) << 24);
                 for (int kk = 0; kk < 16; ++kk)
                     mma_ss(tm, desc(s0 + 8192 + kk * 256, 128, 4096), desc(s0 + 65536 + kk * 256, 128, 256), idn, kk > 0);
+            } else if (mode == 11) {  // K-means MMA1: bf16, A from TMEM, N = 64, 6 instructions
+                const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | ((64u >> 3) << 17) | ((128u >> 4) << 24);
+                for (int p = 0; p < 6; ++p)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tm), "r"(tm + 288 + 8 * p), "l"(desc(s0 + p * 256, 128, 1536)), "r"(idb), "r"((uint32_t)(p > 0)));
+            } else if (mode == 12) {  // K-means MMA2: bf16, A MN-major (LBO 1280 K-groups, SBO 128), B K-major, N = 32, 8 instructions
+                const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | ((32u >> 3) << 17) | ((128u >> 4) << 24);
+                for (int kk = 0; kk < 8; ++kk)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm + 192), "l"(desc(s0 + 8192 + kk * 2560, 1280, 128)), "l"(desc(s0 + 65536 + kk * 256, 128, 2048)), "r"(idb), "r"((uint32_t)(kk > 0)));
+            } else if (mode == 13) {  // MMA1 + MMA2 back to back (one stage of the step)
+                const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | ((64u >> 3) << 17) | ((128u >> 4) << 24);
+                for (int p = 0; p < 6; ++p)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tm), "r"(tm + 288 + 8 * p), "l"(desc(s0 + p * 256, 128, 1536)), "r"(idb), "r"((uint32_t)(p > 0)));
+                const uint32_t id2 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | ((32u >> 3) << 17) | ((128u >> 4) << 24);
+                for (int kk = 0; kk < 8; ++kk)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm + 192), "l"(desc(s0 + 8192 + kk * 2560, 1280, 128)), "l"(desc(s0 + 65536 + kk * 256, 128, 2048)), "r"(id2), "r"((uint32_t)(kk > 0)));
+            } else if (mode == 14) {  // MMA2 with M = 64: bf16 MN-major A, N = 32, 8 instructions
+                const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | ((32u >> 3) << 17) | ((64u >> 4) << 24);
+                for (int kk = 0; kk < 8; ++kk)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tm + 192), "l"(desc(s0 + 8192 + kk * 2560, 1280, 128)), "l"(desc(s0 + 65536 + kk * 256, 128, 2048)), "r"(idb), "r"((uint32_t)(kk > 0)));
+            } else if (mode == 15) {  // MMA1 K = 80: 5 instructions
+                const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | ((64u >> 3) << 17) | ((128u >> 4) << 24);
+                for (int p = 0; p < 5; ++p)
+                    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tm), "r"(tm + 288 + 8 * p), "l"(desc(s0 + p * 256, 128, 1536)), "r"(idb), "r"((uint32_t)(p > 0)));
             } else {                  // kind::f16 (bf16) M128 N32 / N64 K16 x 8
                 const uint32_t NB = mode == 9 ? 32u : 64u;
                 const uint32_t idb = (1u << 4) | (1u << 7) | (1u << 10) | ((NB >> 3) << 17) | ((128u >> 4) << 24);
@@ -91,8 +114,9 @@ int main() {
     cudaMalloc(&o, 16);
     cudaFuncSetAttribute(lat, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
     const char *names[] = {"MMA1 TS x15", "MMA1 SS x15", "MMA2 MN-swz x16", "MMA2-shape K-major x16", "single MMA1 TS",
-                           "x16 N32 4 accumulators", "x16 N64", "x16 N128", "x16 N256", "bf16 x8 N32 K16", "bf16 x8 N64 K16"};
-    for (int m = 0; m < 11; ++m) {
+                           "x16 N32 4 accumulators", "x16 N64", "x16 N128", "x16 N256", "bf16 x8 N32 K16", "bf16 x8 N64 K16", "KM MMA1 bf16 TS N64 x6", "KM MMA2 bf16 MN x8", "KM stage (MMA1+MMA2)",
+                           "MMA2 M64 x8", "MMA1 x5"};
+    for (int m = 0; m < 16; ++m) {
         lat<<<1, 128, 96 * 1024>>>(o, m, 200);
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) { printf("%s: %s\n", names[m], cudaGetErrorString(e)); return 1; }
