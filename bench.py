@@ -5,8 +5,9 @@
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N
 
 A STEP is one pass of the whole hot path over one
-batch of synthetic input resident in HBM, per GPU (weak scaling: rank r owns
-shard r of an N-times larger global problem, seeds offset by r):
+batch of synthetic input resident in HBM.  At N GPUs the same global problem is
+sharded over the ranks (strong scaling, BASELINE.json configs[4]: "k-means
+n=2^26 ... sharded by points"; --weak gives every rank a whole problem):
 
   redomap      f32 add over 2^28 (C4-shaped, 1 GiB)                       A1
   nn_argmin    Rodinia NN argmin redomap, 855,280 (lat,lng) f32 (C2)      A1
@@ -16,9 +17,10 @@ shard r of an N-times larger global problem, seeds offset by r):
                (regimes KG1 / KG2 / KG3 / KG4) and column-major seglen 1024 A4
   seg_scan     f32 add, 2^28 elements, seglen 1024, row-major             A5
   transpose_2d f32 2^14 x 2^14 (C5)                                        A6
-  combine      at N > 1: all_reduce / all_gather + fs_combine of the
-               partials of redomap, nn_argmin, scanomap carries and
-               stream_red (NCCL over NVLink)                               A7
+  combine      at N > 1: ONE collective per exchange (dist.py): all_reduce
+               of the redomap partial, of the packed NN argmin key and of the
+               packed k-means sums + counts; all_gather of the scan totals
+               for the carries (NCCL over NVLink)                          A7
 
 value = algorithmic bytes of all ranks' steps / max-over-ranks device time
 (GB/s, SURVEY.md 8(d) byte counts).  Every input is larger than L2 except
@@ -105,18 +107,31 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ workload
-def build_workload(fs, dev, rank, world, quick):
+def build_workload(fs, dev, rank, world, quick, weak=False):
+    """The step's inputs on this rank.  Strong scaling (default, BASELINE.json configs[4]: the
+    single-GPU problem sharded over the N GPUs): rank r holds shard_range of every global array
+    -- its slice of the 2^28 C4 array (= nseg/N whole rows of every seglen), its records of the
+    855,280 NN records, its points of the 2^26 k-means points, its [2^14/N][2^14] row block of
+    the transpose.  --weak: every rank holds a whole single-GPU problem (seeds offset by rank)."""
     import torch
     import workloads as wl
+    from paper_conf_pldi_henriksenseho17_b200.dist import shard_range
     sh = 4 if quick else 0  # --quick: 16x smaller inputs (for harness checks only)
-    n = (1 << 28) >> sh
+    P, r = (1, 0) if weak else (world, rank)
+    ng = (1 << 28) >> sh
+    lo, hi = shard_range(ng, r, P)
+    n = hi - lo
     W = {}
     W["x"] = wl.device_uniform(n, 5 + 1000 * rank, dev)
-    lat, lng, q = wl.c2_nn(seed=2 + rank)
-    W["lat"], W["lng"], W["q"] = torch.from_numpy(lat).to(dev), torch.from_numpy(lng).to(dev), q
-    W["pts"], W["mem"] = wl.c5_kmeans_shard(rank, dev, n=(1 << 26) >> sh)
+    lat, lng, q = wl.c2_nn(seed=2 + (rank if weak else 0))
+    nlo, nhi = shard_range(lat.size, r, P)
+    W["lat"], W["lng"], W["q"] = torch.from_numpy(lat[nlo:nhi].copy()).to(dev), torch.from_numpy(lng[nlo:nhi].copy()).to(dev), q
+    kg = (1 << 26) >> sh
+    klo, khi = shard_range(kg, r, P)
+    W["pts"], W["mem"] = wl.c5_kmeans_shard(rank, dev, n=khi - klo)
     t = (1 << 14) >> (sh // 2)
-    W["tmat"] = wl.device_uniform((t, t), 6 + 1000 * rank, dev)
+    tlo, thi = shard_range(t, r, P)
+    W["tmat"] = wl.device_uniform((thi - tlo, t), 6 + 1000 * rank, dev)
     # preallocated outputs (no allocation inside the timed region)
     f32 = dict(dtype=torch.float32, device=dev)
     W["o_red"] = torch.empty((), **f32)
@@ -125,20 +140,21 @@ def build_workload(fs, dev, rank, world, quick):
     W["o_sums"] = torch.empty((32, 34), **f32)
     W["o_cnt"] = torch.empty(32, dtype=torch.int32, device=dev)
     W["o_segscan"] = torch.empty(n, **f32)
-    W["o_tr"] = torch.empty((t, t), **f32)
+    W["o_tr"] = torch.empty((t, thi - tlo), **f32)
     W["seglens"] = [32, 1024, 65536, 1 << 20]
     W["o_seg"] = {L: torch.empty(n // L, **f32) for L in W["seglens"]}
     W["o_segcol"] = torch.empty(n // 1024, **f32)
-    W["n"], W["t"] = n, t
-    W["ibase_x"], W["ibase_nn"] = rank * n, rank * lat.size
+    W["n"], W["t"], W["t_rows"] = n, t, thi - tlo
+    W["ibase_x"], W["ibase_nn"] = lo, nlo
+    W["global"] = {"n": ng, "nn": lat.size, "k": kg, "t": t}
     return W
 
 
 def make_step(fs, W, world):
-    """[(name, fn, algorithmic bytes per rank, elements per rank)] for one step."""
-    import torch
+    """[(name, fn, algorithmic bytes per rank, elements per rank)] for one step.  At N > 1 the
+    combines are the multi-GPU layer's single collectives (dist.py)."""
     from paper_conf_pldi_henriksenseho17_b200 import dist as fdist
-    n, t = W["n"], W["t"]
+    n, t, tr = W["n"], W["t"], W["t_rows"]
     nn = W["lat"].numel()
     kn = W["pts"].shape[0]
     multi = world > 1
@@ -146,13 +162,12 @@ def make_step(fs, W, world):
 
     def red():
         if multi:
-            fs.redomap(W["x"], "add", out=W["o_red"])
-            torch.distributed.all_reduce(W["o_red"])
+            fdist.redomap(W["x"], "add")  # local fold + ONE all_reduce
         else:
             fs.redomap(W["x"], "add", out=W["o_red"])
 
     def nn_argmin():
-        if multi:
+        if multi:  # local argmin + packed key + ONE all_reduce MIN
             fdist.redomap(W["lat"], "argmin", ibase=W["ibase_nn"], map="nn_dist", lng=W["lng"], query=W["q"])
         else:
             fs.redomap(W["lat"], "argmin", map="nn_dist", lng=W["lng"], query=W["q"], out=W["o_nn"][0],
@@ -160,19 +175,19 @@ def make_step(fs, W, world):
 
     def scan():
         if multi:
-            fdist.scanomap(W["x"], "add")  # local total + all_gather + carry-in scan (3n)
+            fdist.scanomap(W["x"], "add")  # local total + ONE all_gather + carry-in scan
         else:
             fs.scanomap(W["x"], "add", out=W["o_scan"])
 
     def kmeans():
-        fs.stream_red(W["pts"], W["mem"], 32, sums=W["o_sums"], counts=W["o_cnt"])
         if multi:
-            torch.distributed.all_reduce(W["o_sums"])
-            torch.distributed.all_reduce(W["o_cnt"])
+            fdist.stream_red(W["pts"], W["mem"], 32)  # packed sums + counts, ONE all_reduce
+        else:
+            fs.stream_red(W["pts"], W["mem"], 32, sums=W["o_sums"], counts=W["o_cnt"])
 
     st.append(("redomap_f32_add", red, 4 * n, n))
     st.append(("nn_argmin_redomap", nn_argmin, 8 * nn, nn))
-    st.append(("scanomap_f32_add", scan, (12 if multi else 8) * n, n))
+    st.append(("scanomap_f32_add", scan, 8 * n, n))
     st.append(("stream_red_kmeans_k32_d34", kmeans, (4 * 34 + 4) * kn, kn))
     for L in W["seglens"]:
         st.append((f"seg_reduce_row_L{L}",
@@ -182,7 +197,7 @@ def make_step(fs, W, world):
                                                              out=W["o_segcol"]), 4 * n + 4 * (n // 1024), n))
     st.append(("seg_scan_row_L1024", lambda: fs.seg_scan(W["x"], n // 1024, 1024, "add", out=W["o_segscan"]),
                8 * n, n))
-    st.append(("transpose_2d_f32", lambda: fs.transpose_2d(W["tmat"], out=W["o_tr"]), 8 * t * t, t * t))
+    st.append(("transpose_2d_f32", lambda: fs.transpose_2d(W["tmat"], out=W["o_tr"]), 8 * t * tr, t * tr))
     return st
 
 
@@ -365,6 +380,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--only", default="", help="comma-separated primitive names (profiling aid)")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY 8(f) next-row measurements")
+    ap.add_argument("--weak", action="store_true", help="N > 1: every rank runs a whole single-GPU problem")
     args = ap.parse_args()
     if args.warmup < 3 and not args.quick and not args.only:
         print("bench.py: --warmup must be >= 3", file=sys.stderr)
@@ -395,7 +411,7 @@ def main():
             tdist.init_process_group(backend)
     import paper_conf_pldi_henriksenseho17_b200 as fs
 
-    W = build_workload(fs, dev, rank, world, args.quick)
+    W = build_workload(fs, dev, rank, world, args.quick, weak=args.weak)
     steps = make_step(fs, W, world)
     if args.only:
         keep = set(args.only.split(","))
@@ -441,7 +457,11 @@ def main():
                      "elements_per_s": float(f"{nel / (avg * 1e-3):.4g}"), "bytes": nbytes}
     step_bytes = sum(s[2] for s in steps)
     step_elems = sum(s[3] for s in steps)
-    value = step_bytes * world * K / (total_ms * 1e-3) / GB
+    tot = torch.tensor([step_bytes, step_elems], device=dev, dtype=torch.float64)
+    if world > 1:
+        tdist.all_reduce(tot)  # the whole job's bytes (strong: the global problem; weak: N problems)
+    job_bytes, job_elems = float(tot[0].item()), float(tot[1].item())
+    value = job_bytes * K / (total_ms * 1e-3) / GB
     peak, peak_src = peaks()
     for name in per:
         per[name]["frac_of_peak"] = round(per[name]["GB_s"] / peak, 4)
@@ -478,7 +498,7 @@ def main():
         ems = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
         if world > 1:
             tdist.all_reduce(ems, op=tdist.ReduceOp.MAX)
-        e2e = {"value": round(step_bytes * world * KE / (float(ems.item()) * 1e-3) / GB, 2), "unit": "GB/s",
+        e2e = {"value": round(job_bytes * KE / (float(ems.item()) * 1e-3) / GB, 2), "unit": "GB/s",
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": KE,
                "note": "same algorithmic bytes; pinned host inputs copied in and all outputs copied out every step"}
 
@@ -499,15 +519,18 @@ def main():
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": K,
             "warmup": args.warmup, "ms_per_step": round(total_ms / K, 4), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "weak" if (args.weak and world > 1) else "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
             "config": {"workload": "libfutseg hot-path suite: redomap 2^28 f32, NN argmin 855,280 (C2), scanomap 2^28, "
                                    "k-means stream_red 2^26x34 k=32 (C5), seg_reduce 2^28 L=32/1024/65536/2^20 row + "
                                    "L=1024 col, seg_scan 2^28 L=1024, transpose 2^14^2 f32 (C5)" +
                                    (" [QUICK 1/16 sizes]" if args.quick else ""),
                        "per_rank_bytes_per_step": step_bytes, "per_rank_elements_per_step": step_elems,
                        "l2": "inputs > L2 (126 MB) except NN (6.8 MB), evicted by the ~21 GB rest of each step",
-                       "parallelism": f"dp{world} (weak: one shard per GPU)", "elements_per_s":
-                           float(f"{step_elems * world * K / (total_ms * 1e-3):.4g}")},
+                       "parallelism": (f"dp{world} (weak: a whole single-GPU problem per GPU)" if args.weak else
+                                       f"dp{world} (strong: the single-GPU problem sharded over {world} GPU(s), "
+                                       "BASELINE configs[4])"),
+                       "elements_per_s": float(f"{job_elems * K / (total_ms * 1e-3):.4g}")},
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": per[dom]["GB_s"], "peak": peak, "unit": "GB/s",
                          "frac": round(per[dom]["GB_s"] / peak, 4), "traffic": traffic, "peak_source": peak_src,
                          "bytes_per_launch": per[dom]["bytes"]},

@@ -158,6 +158,42 @@ fs_status fs_scanomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void 
 fs_status fs_combine(fs_opdesc op, const void *parts, const int64_t *part_idx, int64_t P, void *out,
                      int64_t *out_idx, void *stream);
 
+/* ---------------------------------------------------------------- cross-GPU exchange */
+/* The per-GPU halves of the multi-GPU combine (north_star "combined with one
+ * NCCL allreduce"): a rank's partial results are packed into ONE buffer of one reducible type
+ * so that each exchange of the multi-GPU layer is a single collective, then unpacked.
+ *
+ * fs_argmin_pack: for ARGMIN partials (value, global index) of dtype I32 / F32, keys[i] =
+ *   int64 whose signed order is the lexicographic (value, index) order of reading R3 (index -1,
+ *   "no element", orders last): one all_reduce MIN over the ranks is the exact global argmin.
+ *   Requires -1 <= idx < 2^32 - 1.  For I64 values keys is [n][2] = (value, index) records,
+ *   to be all_gathered.
+ * fs_argmin_unpack: I32 / F32: decodes ONE reduced key (P must be 1) into value / idx (the
+ *   neutral element (+inf or INT32_MAX, -1) when no rank had an element).  I64: folds the P
+ *   gathered records in rank order with R3's operator.
+ *   values, idx, keys: device pointers; no workspace; FS_ERR_SIZE, _NULL, _UNSUPPORTED, _ALIAS. */
+fs_status fs_argmin_pack(int32_t dtype, const void *values, const int64_t *idx, int64_t n, int64_t *keys,
+                         void *stream);
+fs_status fs_argmin_unpack(int32_t dtype, const int64_t *keys, int64_t P, void *value, int64_t *idx,
+                           void *stream);
+/* fs_partials_pack: packed[0 .. k*w) = sums, [k*w .. k*w+k) = counts (0 when counts is NULL),
+ *   packed[k*w+k] = *extra (0 when NULL, e.g. the k-means delta): 8-byte elements, f64 for
+ *   F32 sums (exact widening; counts exact below 2^53) and int64 for I32 / I64 sums (I32
+ *   sign-extended).  One all_reduce SUM of the packed buffer combines the ranks' partials
+ *   (Fig 4c's map(+) across chunks, L526-531); integer sums stay exact modulo 2^32 / 2^64 (R1).
+ * fs_partials_unpack: the inverse after the reduction: F32 sums rounded once from the f64
+ *   total, I32 sums the low 32 bits, counts / extra converted back.  sums [k][w] of dtype,
+ *   counts [k] int32, extra int64; counts / extra may be NULL. */
+fs_status fs_partials_pack(int32_t dtype, const void *sums, const int32_t *counts, const int64_t *extra, int64_t k,
+                           int64_t w, void *packed, void *stream);
+fs_status fs_partials_unpack(int32_t dtype, const void *packed, int64_t k, int64_t w, void *sums, int32_t *counts,
+                             int64_t *extra, void *stream);
+/* fs_copy_2d: dst[r*dst_ld + c] = src[r*src_ld + c] for r < rows, c < cols, elements of
+ *   elem_bytes (4 or 8): the column-block gather of the distributed transpose (rearrange (1,0)
+ *   of a row-sharded matrix, L1389-1393).  src and dst must not overlap (FS_ERR_ALIAS). */
+fs_status fs_copy_2d(int32_t elem_bytes, const void *src, int64_t src_ld, int64_t rows, int64_t cols, void *dst,
+                     int64_t dst_ld, void *stream);
+
 /* ---------------------------------------------------------------- stream_red */
 /* The K-means centre update (Fig 4c; Sec. 2.4; L1649):
  *   sums[c][j] = sum of vals[i][j] over i with keys[i] == c      (c < k, j < w)

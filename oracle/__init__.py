@@ -35,10 +35,11 @@ LAYOUTS = {"row": 0, "col": 1}
 def build(force: bool = False) -> str:
     """Compile oracle.c with gcc (no fast-math, no FP contraction)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = f"{_LIB}.{os.getpid()}.tmp"  # concurrent builders (spawned test ranks) each replace atomically
         subprocess.check_call([
             "gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-std=c11",
-            "-shared", "-fPIC", _SRC, "-o", _LIB + ".tmp", "-lm"])
-        os.replace(_LIB + ".tmp", _LIB)
+            "-shared", "-fPIC", _SRC, "-o", tmp, "-lm"])
+        os.replace(tmp, _LIB)
     return _LIB
 
 

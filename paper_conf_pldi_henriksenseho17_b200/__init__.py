@@ -24,7 +24,7 @@ import torch
 
 __all__ = [
     "FutsegError", "redomap", "scanomap", "stream_red", "seg_reduce", "seg_scan", "transpose_2d",
-    "combine", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "last_seg_regime", "force_seg_regime", "library_path", "version",
+    "combine", "argmin_pack", "argmin_unpack", "partials_pack", "partials_unpack", "copy_2d", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "check_device_error", "seg_regime", "last_seg_regime", "force_seg_regime", "library_path", "version",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -81,6 +81,11 @@ _SIG = {
     "fs_scan_reduce": [_I, _I, _I, _P, _L, _P, _P, ctypes.c_size_t, _P],
     "fs_kmeans_finish": [_P, _P, _P, _L, _L, _P, _P],
     "fs_check_device_error": [_P, _P],
+    "fs_argmin_pack": [_I, _P, _P, _L, _P, _P],
+    "fs_argmin_unpack": [_I, _P, _L, _P, _P, _P],
+    "fs_partials_pack": [_I, _P, _P, _P, _L, _L, _P, _P],
+    "fs_partials_unpack": [_I, _P, _L, _L, _P, _P, _P, _P],
+    "fs_copy_2d": [_I, _P, _L, _L, _L, _P, _L, _P],
     "fs_seg_regime": [_I, fs_opdesc, _L, _L, _I],
     "fs_force_seg_regime": [_I],
     "fs_last_seg_regime": [],
@@ -230,7 +235,7 @@ def scanomap(x, op: str = "add", map: str = "id", lng=None, query=(0.0, 0.0), ca
     return (out, out_idx) if op == "argmin" else out
 
 
-def combine(parts, op: str = "add", part_idx=None, width: int = 1):
+def combine(parts, op: str = "add", part_idx=None, width: int = 1, out=None, out_idx=None):
     """parts[0] (+) ... (+) parts[P-1] (the final combine of per-chunk / per-GPU partials)."""
     parts = _dev(parts, "parts")
     dt = _dt(parts)
@@ -238,11 +243,70 @@ def combine(parts, op: str = "add", part_idx=None, width: int = 1):
     if op == "vadd":
         width = parts.shape[1]
     o = _op(op, dt, width)
-    out = torch.empty(width if op == "vadd" else (), dtype=parts.dtype, device=parts.device)
-    out_idx = torch.empty((), dtype=torch.int64, device=parts.device) if op == "argmin" else None
+    if out is None:
+        out = torch.empty(width if op == "vadd" else (), dtype=parts.dtype, device=parts.device)
+    if op == "argmin" and out_idx is None:
+        out_idx = torch.empty((), dtype=torch.int64, device=parts.device)
     _ok(_lib.fs_combine(o, _ptr(parts), _ptr(part_idx), P, ctypes.c_void_p(out.data_ptr()),
                         _ptr(out_idx) if out_idx is not None else None, _stream(parts.device)), "fs_combine")
     return (out, out_idx) if op == "argmin" else out
+
+
+def argmin_pack(values, idx, out=None):
+    """ARGMIN partials -> int64 keys whose signed MIN is the R3 argmin (i32 / f32: [n] keys;
+    i64: [n][2] (value, index) records for an all_gather).  One collective per exchange."""
+    values, idx = _dev(values, "values"), _dev(idx, "idx")
+    dt = _dt(values)
+    n = values.numel()
+    if out is None:
+        out = torch.empty((n, 2) if dt == FS_I64 else n, dtype=torch.int64, device=values.device)
+    _ok(_lib.fs_argmin_pack(dt, _ptr(values), _ptr(idx), n, _ptr(out), _stream(values.device)), "fs_argmin_pack")
+    return out
+
+
+def argmin_unpack(keys, dtype, P: int = 1, out=None, out_idx=None):
+    """The reduced key (i32 / f32, P = 1) or the P gathered records (i64) -> (value, index)."""
+    keys = _dev(keys, "keys")
+    dt = _DT[dtype]
+    if out is None:
+        out = torch.empty((), dtype=dtype, device=keys.device)
+    if out_idx is None:
+        out_idx = torch.empty((), dtype=torch.int64, device=keys.device)
+    _ok(_lib.fs_argmin_unpack(dt, _ptr(keys), P, ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(out_idx.data_ptr()),
+                              _stream(keys.device)), "fs_argmin_unpack")
+    return out, out_idx
+
+
+def partials_pack(sums, counts=None, extra=None, out=None):
+    """sums [k][w] (+ counts [k], + one extra int64 such as delta) -> ONE buffer of k*w + k + 1
+    f64 (f32 sums) or int64 (integer sums) for a single all_reduce SUM."""
+    sums = _dev(sums, "sums")
+    dt = _dt(sums)
+    k, w = (sums.shape[0], sums.shape[1]) if sums.dim() == 2 else (sums.numel(), 1)
+    if out is None:
+        out = torch.empty(k * w + k + 1, dtype=torch.float64 if dt == FS_F32 else torch.int64, device=sums.device)
+    _ok(_lib.fs_partials_pack(dt, _ptr(sums), _ptr(counts), _ptr(extra), k, w, ctypes.c_void_p(out.data_ptr()),
+                              _stream(sums.device)), "fs_partials_pack")
+    return out
+
+
+def partials_unpack(packed, sums, counts=None, extra=None):
+    """Inverse of partials_pack after the reduction, into the given sums / counts / extra."""
+    packed, sums = _dev(packed, "packed"), _dev(sums, "sums")
+    dt = _dt(sums)
+    k, w = (sums.shape[0], sums.shape[1]) if sums.dim() == 2 else (sums.numel(), 1)
+    _ok(_lib.fs_partials_unpack(dt, ctypes.c_void_p(packed.data_ptr()), k, w, _ptr(sums), _ptr(counts), _ptr(extra),
+                                _stream(sums.device)), "fs_partials_unpack")
+    return sums, counts, extra
+
+
+def copy_2d(src, rows: int, cols: int, src_ld: int, dst, dst_ld: int):
+    """dst[r][c] = src[r][c] for r < rows, c < cols with leading dimensions src_ld / dst_ld
+    (elements; tensors are flat views starting at element (0, 0))."""
+    src, dst = _dev(src, "src"), _dev(dst, "dst")
+    _ok(_lib.fs_copy_2d(src.element_size(), _ptr(src), src_ld, rows, cols, _ptr(dst), dst_ld, _stream(src.device)),
+        "fs_copy_2d")
+    return dst
 
 
 def nn_knn(lat, lng, query, kk: int, out_dist=None, out_idx=None):

@@ -499,6 +499,71 @@ fs_status fs_scan_reduce(int32_t scan_op, int32_t red_op, int32_t dtype, const v
     return scan_reduce_run(red_op, dtype, in, n, out, ws, S(stream));
 }
 
+// ------------------------------------------------------------ multi-GPU exchange helpers
+fs_status fs_argmin_pack(int32_t dtype, const void *values, const int64_t *idx, int64_t n, int64_t *keys,
+                         void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (n < 0) return FS_ERR_SIZE;
+    if (n == 0) return FS_OK;
+    if (!values || !idx || !keys) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype), kb = n * (dtype == FS_I64 ? 16 : 8);
+    if (!aligned_to(values, es) || !aligned_to(idx, 8) || !aligned_to(keys, 8)) return FS_ERR_UNSUPPORTED;
+    if (overlaps(keys, kb, values, n * es) || overlaps(keys, kb, idx, n * 8)) return FS_ERR_ALIAS;
+    return argmin_pack_run(dtype, values, idx, n, keys, S(stream));
+}
+
+fs_status fs_argmin_unpack(int32_t dtype, const int64_t *keys, int64_t P, void *value, int64_t *idx, void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (P < 0 || (dtype != FS_I64 && P != 1)) return FS_ERR_SIZE;
+    if ((P > 0 && !keys) || !value || !idx) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype), kb = P * (dtype == FS_I64 ? 16 : 8);
+    if ((keys && !aligned_to(keys, 8)) || !aligned_to(value, es) || !aligned_to(idx, 8)) return FS_ERR_UNSUPPORTED;
+    if (overlaps(value, es, keys, kb) || overlaps(idx, 8, keys, kb)) return FS_ERR_ALIAS;
+    return argmin_unpack_run(dtype, keys, P, value, idx, S(stream));
+}
+
+fs_status fs_partials_pack(int32_t dtype, const void *sums, const int32_t *counts, const int64_t *extra, int64_t k,
+                           int64_t w, void *packed, void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (k < 0 || w < 0 || mul_overflows(k, w)) return FS_ERR_SIZE;
+    if (!packed || (k * w > 0 && !sums)) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype), pb = (k * w + k + 1) * 8;
+    if ((sums && !aligned_to(sums, es)) || (counts && !aligned_to(counts, 4)) || (extra && !aligned_to(extra, 8)) ||
+        !aligned_to(packed, 8))
+        return FS_ERR_UNSUPPORTED;
+    if (overlaps(packed, pb, sums, k * w * es) || overlaps(packed, pb, counts, k * 4) || overlaps(packed, pb, extra, 8))
+        return FS_ERR_ALIAS;
+    return partials_pack_run(dtype, sums, counts, extra, k * w, k, packed, S(stream));
+}
+
+fs_status fs_partials_unpack(int32_t dtype, const void *packed, int64_t k, int64_t w, void *sums, int32_t *counts,
+                             int64_t *extra, void *stream) {
+    if (!valid_dtype(dtype)) return FS_ERR_UNSUPPORTED;
+    if (k < 0 || w < 0 || mul_overflows(k, w)) return FS_ERR_SIZE;
+    if (!packed || (k * w > 0 && !sums)) return FS_ERR_NULL;
+    const int64_t es = (int64_t)dtype_size(dtype), pb = (k * w + k + 1) * 8;
+    if ((sums && !aligned_to(sums, es)) || (counts && !aligned_to(counts, 4)) || (extra && !aligned_to(extra, 8)) ||
+        !aligned_to(packed, 8))
+        return FS_ERR_UNSUPPORTED;
+    if (overlaps(packed, pb, sums, k * w * es) || overlaps(packed, pb, counts, k * 4) || overlaps(packed, pb, extra, 8))
+        return FS_ERR_ALIAS;
+    return partials_unpack_run(dtype, packed, k * w, k, sums, counts, extra, S(stream));
+}
+
+fs_status fs_copy_2d(int32_t elem_bytes, const void *src, int64_t src_ld, int64_t rows, int64_t cols, void *dst,
+                     int64_t dst_ld, void *stream) {
+    if (elem_bytes != 4 && elem_bytes != 8) return FS_ERR_UNSUPPORTED;
+    if (rows < 0 || cols < 0 || src_ld < cols || dst_ld < cols || mul_overflows(rows, src_ld) ||
+        mul_overflows(rows, dst_ld))
+        return FS_ERR_SIZE;
+    if (rows * cols == 0) return FS_OK;
+    if (!src || !dst) return FS_ERR_NULL;
+    if (!aligned_to(src, elem_bytes) || !aligned_to(dst, elem_bytes)) return FS_ERR_UNSUPPORTED;
+    const int64_t sb = ((rows - 1) * src_ld + cols) * elem_bytes, db = ((rows - 1) * dst_ld + cols) * elem_bytes;
+    if (overlaps(dst, db, src, sb)) return FS_ERR_ALIAS;
+    return copy_2d_run(elem_bytes, src, src_ld, rows, cols, dst, dst_ld, S(stream));
+}
+
 // ------------------------------------------------------------ utilities
 fs_status fs_check_device_error(void *ws, void *stream) {
     if (!ws) return FS_ERR_NULL;

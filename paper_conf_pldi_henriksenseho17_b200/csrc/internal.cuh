@@ -111,6 +111,15 @@ size_t scan_reduce_ws(int dt);
 fs_status scan_reduce_run(int red, int dt, const void *x, int64_t n, void *out, void *ws, cudaStream_t st);
 fs_status kmeans_finish_run(const float *sums, const int32_t *counts, const float *cen, int64_t k, int64_t d,
                             float *new_cen, cudaStream_t st);
+// exchange.cu (the multi-GPU layer's one-collective exchanges)
+fs_status argmin_pack_run(int dt, const void *val, const int64_t *idx, int64_t n, int64_t *key, cudaStream_t st);
+fs_status argmin_unpack_run(int dt, const int64_t *key, int64_t P, void *val, int64_t *idx, cudaStream_t st);
+fs_status partials_pack_run(int dt, const void *sums, const int32_t *counts, const int64_t *extra, int64_t kw,
+                            int64_t k, void *packed, cudaStream_t st);
+fs_status partials_unpack_run(int dt, const void *packed, int64_t kw, int64_t k, void *sums, int32_t *counts,
+                              int64_t *extra, cudaStream_t st);
+fs_status copy_2d_run(int eb, const void *src, int64_t sld, int64_t rows, int64_t cols, void *dst, int64_t dld,
+                      cudaStream_t st);
 // transpose.cu
 fs_status transpose_run(int dt, const void *in, int64_t rows, int64_t cols, void *out, cudaStream_t st);
 
