@@ -103,6 +103,26 @@ _lib.fs_launch_count.restype = ctypes.c_uint64
 
 C = _lib  # raw C ABI (ctypes), for callers that manage their own device pointers
 
+# NVTX ranges (tracing): FUTSEG_NVTX=1 wraps every primitive of this module in an
+# NVTX range named "futseg.<primitive>" (visible in nsys / ncu --nvtx); off by default so that
+# the ~1 us of range push/pop never perturbs a timed region.
+_NVTX = os.environ.get("FUTSEG_NVTX", "0") not in ("", "0")
+
+
+def _traced(fn):
+    if not _NVTX:
+        return fn
+    import functools
+
+    @functools.wraps(fn)
+    def wrapper(*args, **kw):
+        torch.cuda.nvtx.range_push("futseg." + fn.__name__)
+        try:
+            return fn(*args, **kw)
+        finally:
+            torch.cuda.nvtx.range_pop()
+    return wrapper
+
 
 class FutsegError(RuntimeError):
     def __init__(self, status: int, where: str):
@@ -489,3 +509,9 @@ def last_seg_regime() -> int:
 
 def force_seg_regime(regime: int):
     _ok(_lib.fs_force_seg_regime(int(regime)), "fs_force_seg_regime")
+
+
+for _name in ("redomap", "scanomap", "combine", "argmin_pack", "argmin_unpack", "partials_pack", "partials_unpack",
+              "copy_2d", "nn_knn", "kmeans_step", "kmeans_finish", "seg_map_reduce", "scan_reduce", "stream_red",
+              "seg_reduce", "seg_scan", "transpose_2d"):
+    globals()[_name] = _traced(globals()[_name])

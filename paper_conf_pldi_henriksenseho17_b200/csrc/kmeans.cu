@@ -339,9 +339,9 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             mbar_init(&B.raw_empty[s], 4);
         }
         for (int s = 0; s < kKmNA; ++s) {
-            mbar_init(&B.a1full[s], 4);
+            mbar_init(&B.a1full[s], 128);  // every convert thread (its |x|^2 store and TMEM rows)
             mbar_init(&B.d1full[s], 1);
-            mbar_init(&B.slotfree[s], 4);
+            mbar_init(&B.slotfree[s], 128);  // every decide thread (its D1 row and |x|^2 read)
         }
         for (int s = 0; s < NX; ++s) {
             mbar_init(&B.ohfull[s], 4);
@@ -445,11 +445,9 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
             fence_proxy_async();
             tc_fence_before();
+            km_arrive(&B.a1full[sa]);
             __syncwarp();
-            if (lane == 0) {
-                if (full) km_arrive(&B.raw_empty[s % NR]);
-                km_arrive(&B.a1full[sa]);
-            }
+            if (lane == 0 && full) km_arrive(&B.raw_empty[s % NR]);
             KM_TRACE(s, 2);
         }
     } else if (warp < kKmWarpProd) {
@@ -507,8 +505,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             const float nrm = B.nrm[sa][r];
             KM_TRACE(s, 4);
             tc_fence_before();
-            __syncwarp();
-            if (lane == 0) km_arrive(&B.slotfree[sa]);
+            km_arrive(&B.slotfree[sa]);
             float m1 = fminf(dd[0], dd[1]);
 #pragma unroll
             for (int c = 2; c + 1 < NC; c += 2) m1 = fmin3(m1, dd[c], dd[c + 1]);

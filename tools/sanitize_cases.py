@@ -71,5 +71,38 @@ fs.seg_map_reduce(xb, 600, 8192, 1.0, "max")
 xk = cu(workloads.mixed(600 * 12_289 + 1, 9, np.float32))
 fs.seg_scan(xk[: 600 * 12_289], 600, 12_289, "add")
 fs.seg_scan(xk[1:], 600, 12_289, "argmin")
+# round 2: every seg_scan regime of the plan (fs::seg_scan_plan), forced where applicable --
+# KS0-BIG (power-of-two rows of 2-8 CTA steps), KS3 (several rows per CTA, one row per CTA,
+# 8-byte, misaligned views), KS2, the flat slab scan per row, the look-back scan
+xr = cu(workloads.mixed(150 * 12_288 + 8, 10, np.float32))
+xri = cu(workloads.mixed(150 * 12_288 + 8, 10, np.int64))
+for reg in (5, 7, 8, 9, 10, 11, 12):
+    fs.force_seg_regime(reg)
+    for nseg, L in ((64, 2048), (17, 8192), (300, 33), (7, 1000), (3, 16_384), (150, 12_288), (777, 3)):
+        fs.seg_scan(xr[: nseg * L], nseg, L, "add")
+        fs.seg_scan(xri[: nseg * L], nseg, L, "min")
+    fs.force_seg_regime(-1)
+for nseg, L, off in ((64, 1000, 1), (7, 4097, 1), (300, 33, 3)):
+    fs.seg_scan(xr[off: off + nseg * L], nseg, L, "max")   # KS3 on misaligned views
+    fs.seg_scan(xri[off: off + nseg * L], nseg, L, "add")
+xl = cu(workloads.mixed(2 * (1 << 20), 11, np.float32))
+fs.force_seg_regime(12)
+fs.seg_scan(xl, 2, 1 << 20, "add")  # the flat per-row slab scan
+fs.force_seg_regime(-1)
+# the tcgen05 k-means step (TMA ring, TMEM A, both MMAs, d = 34 specialisation and run-time d,
+# a partial last stage) and the multi-GPU exchange kernels
+pts, _ = workloads.c3_kmeans(n=40_011, d=34, k=32)
+fs.kmeans_step(cu(pts), cu(pts[:32].copy()), prev=cu(workloads.ints(40_011, 3, 0, 32)))
+pts, _ = workloads.c3_kmeans(n=9_999, d=40, k=17)
+fs.kmeans_step(cu(pts), cu(pts[:17].copy()))
+v = cu(workloads.mixed(9, 12, np.float32))
+i = cu(np.arange(9, dtype=np.int64))
+k = fs.argmin_pack(v, i)
+fs.argmin_unpack(k[:1], torch.float32)
+k8 = fs.argmin_pack(cu(workloads.mixed(9, 13, np.int64)), i)
+fs.argmin_unpack(k8, torch.int64, P=9)
+pk = fs.partials_pack(cu(workloads.mixed((5, 7), 14, np.float32)), cu(np.arange(5, dtype=np.int32)))
+fs.partials_unpack(pk, torch.empty((5, 7), device="cuda"), torch.empty(5, dtype=torch.int32, device="cuda"))
+fs.copy_2d(x[1:], 33, 17, 41, torch.empty(33 * 19 + 1, device="cuda")[1:], 19)
 torch.cuda.synchronize()
 print("sanitize cases done")
