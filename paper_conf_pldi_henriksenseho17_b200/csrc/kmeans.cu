@@ -191,6 +191,7 @@ __device__ __forceinline__ float km_exact(const float *x, const float *c, int d)
 // FUTSEG_KM_TRACE is set; [stage][8]: convert begin / ready / end, decide begin / ready / end,
 // MMA1 issue, MMA2 issue.
 __device__ long long *g_km_trace = nullptr;
+__device__ int g_km_trace_cta = 0;
 
 #define KM_TRACE(s, e)                                                                   \
     do {                                                                                 \
@@ -305,7 +306,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         reinterpret_cast<unsigned char *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int d = DT > 0 ? DT : d_rt;  // DT > 0: the width is a compile-time constant (C3 / C5: 34)
-    long long *const trace = blockIdx.x == 0 ? g_km_trace : nullptr;  // debug tracing (normally null)
+    long long *const trace = (int)blockIdx.x == g_km_trace_cta ? g_km_trace : nullptr;  // debug tracing (normally null)
     const int skip = g_km_skip;                                        // debug timing switches (0)
     constexpr bool EVEN = DT > 0 && DT % 2 == 0;
     const KmGeom G(d);
@@ -456,9 +457,9 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         const int dg = (warp - kKmWarpDecide) >> 2, wl = warp & 3, r = wl * 32 + lane;
         const uint32_t t_lane = (uint32_t)(wl * 32) << 16;
         const float cmax2 = B.cmax2;
-        float *acc_tot = s_acc + r * NC;  // this thread's M row of the D2 totals (group 0)
+        float *acc_tot = s_acc + r;  // this thread's M row of the D2 totals (group 0): [c][128], conflict-free
         if (dg == 0)
-            for (int c = 0; c < NC; ++c) acc_tot[c] = 0.f;
+            for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = 0.f;
         int ohpos[kKmNXMax];
 #pragma unroll
         for (int q = 0; q < kKmNXMax; ++q) ohpos[q] = -1;
@@ -471,7 +472,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             float v[32];
             tmem_ld32(tD2 + t_lane + (uint32_t)(b2 * NC), v);
 #pragma unroll
-            for (int c = 0; c < NC; ++c) acc_tot[c] = __fadd_rn(acc_tot[c], v[c]);
+            for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = __fadd_rn(acc_tot[c * kKmRows], v[c]);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) km_arrive(&B.d2free[b2]);
@@ -551,7 +552,11 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             __syncwarp();
             if (lane == 0) km_arrive(&B.ohfull[sx]);
             KM_TRACE(s, 5);
-            if (dg == 0 && flushed < nseg2 && (flushed + 1) * kKmSeg + 1 <= s) flush();  // group 0 owns D2
+            // group 0 owns D2: move a finished buffer to the totals once its last MMA2 has completed
+            // (tested, never waited for here -- a blocking wait stalled the pipeline every 16 stages)
+            if (dg == 0 && flushed < nseg2 && (flushed + 1) * kKmSeg <= s &&
+                km_test(&B.d2full[flushed & 1], (unsigned)((flushed >> 1) & 1)))
+                flush();
         }
         if (dg == 0)
             while (flushed < nseg2) flush();
@@ -561,7 +566,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         // the partial
         km_bar_sync(1, 4 * kKmDc * 32);
         if (dg == 0)
-            for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c];
+            for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c * kKmRows];
     } else if (warp == kKmWarpProd) {
         // =============================== producer: TMA bulk copies of full stages
         if (lane == 0) {
@@ -731,6 +736,8 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
         if (e && !tr) cudaMalloc(&tr, 16 * 8 * 8192);
         long long *p = e ? tr : nullptr;
         cudaMemcpyToSymbolAsync(g_km_trace, &p, sizeof(p), 0, cudaMemcpyHostToDevice, st);
+        static int cta = e ? atoi(e) : 0;
+        cudaMemcpyToSymbolAsync(g_km_trace_cta, &cta, sizeof(cta), 0, cudaMemcpyHostToDevice, st);
         static int skip = getenv("FUTSEG_KM_SKIP") ? atoi(getenv("FUTSEG_KM_SKIP")) : 0;
         cudaMemcpyToSymbolAsync(g_km_skip, &skip, sizeof(skip), 0, cudaMemcpyHostToDevice, st);
     }

@@ -17,3 +17,19 @@ for _ in range(10):
 ms = float(np.median(ts))
 byt = pts.shape[0] * (34 * 4 + 8)
 print(f"mode={os.environ.get('FUTSEG_KM_DEBUG','0')} C5 kmeans_step: {ms:.3f} ms  {byt / ms / 1e6:.1f} GB/s  frac {byt / ms / 1e6 / 6546.9:.3f}", flush=True)
+# SM clock / power while the step runs back to back (NVML), to see whether the tensor-core-heavy
+# kernel runs under the power cap
+import threading, pynvml
+pynvml.nvmlInit()
+h = pynvml.nvmlDeviceGetHandleByIndex(0)
+samples, stop = [], threading.Event()
+def samp():
+    while not stop.is_set():
+        samples.append((pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM), pynvml.nvmlDeviceGetPowerUsage(h) / 1000,
+                        pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)))
+        stop.wait(0.02)
+th = threading.Thread(target=samp); th.start()
+for _ in range(300): f()
+torch.cuda.synchronize(); stop.set(); th.join()
+cl = sorted(s[0] for s in samples); pw = sorted(s[1] for s in samples)
+print(f"clocks during 300 steps: median {cl[len(cl)//2]} MHz (min {cl[0]}), power median {pw[len(pw)//2]:.0f} W max {pw[-1]:.0f} W, reasons {sorted(set(s[2] for s in samples))}")
