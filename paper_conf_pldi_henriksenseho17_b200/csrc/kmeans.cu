@@ -233,10 +233,13 @@ __device__ int g_km_skip = 0;  // debug: bit 0 skips the MMA2 instructions, bit 
 // lane of the calling thread, K-major pairs: [a1 | 1 1 1 | 0..] then [a2 | 0..], KP columns each)
 // and as the MMA2 A operand (shared memory, MN-major: the row is the K index, a1 rows 0..d-1, the
 // count row d, a2 rows JB..JB+d-1).  Returns |x|^2 (f32).
-template <bool FULL, bool EVEN>
+// PK (even compile-time d): MMA1's A packed as [a1 (d) | a2 (d) | 1 1 1 | 0] in K1 = roundup16(2d + 3)
+// columns (5 instructions at d = 34 instead of 6); otherwise [a1 | 1 1 1 | 0] [a2 | 0], KP each.
+template <bool FULL, bool EVEN, int PK>
 __device__ __forceinline__ float km_convert_row(const float *src, int d, bool valid, const KmGeom &G, int qd,
                                                 uint32_t ta, unsigned char *xr, int skip) {
     float nrm = 0.f;
+    uint32_t a2w[PK > 0 ? PK / 2 + 8 : 1];  // PK: the a2 pairs (+ the last a1 pairs), stored after the loop
 #pragma unroll
     for (int q = 0; q < 3; ++q) {  // 16 columns per chunk (KP <= 48)
         if (16 * q < G.KP) {
@@ -278,7 +281,12 @@ __device__ __forceinline__ float km_convert_row(const float *src, int d, bool va
                     wx[t] |= ((j0 == d && valid) ? 0x3F80u : 0u) | ((j1 == d && valid) ? 0x3F800000u : 0u);
                 }
             }
-            if (!(skip & 4)) {
+            if (PK > 0) {
+#pragma unroll
+                for (int t = 0; t < 8; ++t)
+                    if (8 * q + t < PK / 2) a2w[8 * q + t] = w2[t];
+                if (8 * q + 8 <= PK / 2) tmem_st8u(ta + 8 * q, w1);  // whole chunks of a1 pairs
+            } else if (!(skip & 4)) {
                 tmem_st8u(ta + 8 * q, wt);
                 tmem_st8u(ta + G.KP / 2 + 8 * q, w2);
             }
@@ -290,6 +298,24 @@ __device__ __forceinline__ float km_convert_row(const float *src, int d, bool va
                 *reinterpret_cast<uint4 *>(xr + (G.JB / 8 + 2 * q) * 128) = make_uint4(w2[0], w2[1], w2[2], w2[3]);
             if (16 * q + 8 < d)
                 *reinterpret_cast<uint4 *>(xr + (G.JB / 8 + 2 * q + 1) * 128) = make_uint4(w2[4], w2[5], w2[6], w2[7]);
+            if (PK > 0 && 8 * q + 8 > PK / 2 && 8 * q < PK / 2) {  // the chunk holding the last a1 pairs
+#pragma unroll
+                for (int t = 0; t < 8; ++t)
+                    if (8 * q + t < PK / 2) a2w[PK / 2 + 1 + t] = w1[t];  // parked past the a2 pairs
+            }
+        }
+    }
+    if (PK > 0) {  // words [8 (PK/2 / 8), K1 / 2): remaining a1 pairs, a2 pairs, augmentation, zeros
+        constexpr int H = PK / 2, W0 = H / 8 * 8, K1W = (2 * PK + 3 + 15) / 16 * 8;
+#pragma unroll
+        for (int w0 = W0; w0 < K1W; w0 += 8) {
+            uint32_t v[8];
+#pragma unroll
+            for (int t = 0; t < 8; ++t) {
+                const int w = w0 + t;
+                v[t] = w < H ? a2w[H + 1 + (w - W0)] : (w < 2 * H ? a2w[w - H] : (w == 2 * H ? 0x3F803F80u : (w == 2 * H + 1 ? 0x3F80u : 0u)));
+            }
+            tmem_st8u(ta + w0, v);
         }
     }
     return nrm;
@@ -309,7 +335,9 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     long long *const trace = (int)blockIdx.x == g_km_trace_cta ? g_km_trace : nullptr;  // debug tracing (normally null)
     const int skip = g_km_skip;                                        // debug timing switches (0)
     constexpr bool EVEN = DT > 0 && DT % 2 == 0;
+    constexpr int PKD = EVEN ? DT : 0;  // packed MMA1 K layout (compile-time even d)
     const KmGeom G(d);
+    const int K1 = PKD > 0 ? (2 * PKD + 3 + 15) / 16 * 16 : 2 * G.KP;  // MMA1 K
     constexpr int N1 = 2 * NC;  // MMA1 N: (centre, b piece)
     // ---- shared memory carve-up
     const uint32_t raw_bytes = (uint32_t)(kKmRows * d * 4);
@@ -317,7 +345,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     const uint32_t x2_bytes = (uint32_t)G.x2_bytes();
     constexpr uint32_t oh_bytes = NC / 8 * 2048;           // [centre group][16 row chunks][8 x 16 B]
     const uint32_t LB2 = (uint32_t)(G.NG * 128);           // MMA2 A: K-group (8 rows) stride
-    const uint32_t SB1 = (uint32_t)(2 * G.KP / 8 * 128);  // MMA1 B: n-group stride (K1 = 2 KP)
+    const uint32_t SB1 = (uint32_t)(2 * G.KP / 8 * 128);  // MMA1 B: n-group stride (room for K1 <= 2 KP)
     unsigned char *raw = smem;                              // [NR][raw_slot]
     unsigned char *x2 = raw + NR * raw_slot;                // [NX][x2_bytes] + 1 KB (MMA2 M read-beyond)
     unsigned char *oh = x2 + NX * x2_bytes + 1024;          // [NX][oh_bytes]
@@ -371,15 +399,25 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     // pieces q1 q2 q3 in columns d, d+1, d+2 of the a1 half; n >= NC is centre n - NC with the b2
     // piece.  The a2 half of K (k >= KP) repeats the b piece without |c|^2.  Padding centres have
     // |c|^2 = 2^100 (finite: 0 * it stays 0), so they are never candidates.
-    for (int e = tid; e < N1 * 2 * G.KP; e += kKmThreads) {
-        const int nn = e / (2 * G.KP), kk = e - nn * (2 * G.KP);
-        const int c = nn < NC ? nn : nn - NC, piece = nn < NC ? 0 : 1, j = kk < G.KP ? kk : kk - G.KP;
+    for (int e = tid; e < N1 * K1; e += kKmThreads) {
+        const int nn = e / K1, kk = e - nn * K1;
+        const int c = nn < NC ? nn : nn - NC, piece = nn < NC ? 0 : 1;
+        // the x column (or augmentation slot) this K index multiplies
+        int j, aug;
+        if (PKD > 0) {
+            j = kk < 2 * d ? (kk < d ? kk : kk - d) : -1;
+            aug = kk >= 2 * d && kk <= 2 * d + 2 ? kk - 2 * d : -1;
+        } else {
+            const int jj = kk < G.KP ? kk : kk - G.KP;
+            j = jj < d ? jj : -1;
+            aug = (kk < G.KP && jj >= d && jj <= d + 2) ? jj - d : -1;
+        }
         float v = 0.f;
-        if (j < d) {
+        if (j >= 0) {
             const float b = c < k ? -2.f * cen_s[c * kKmMaxD + j] : 0.f;
             const float p1 = bfr(b);
             v = piece == 0 ? p1 : bfr(__fsub_rn(b, p1));
-        } else if (kk < G.KP && piece == 0 && j <= d + 2) {
+        } else if (aug >= 0 && piece == 0) {
             float c2 = 0x1p100f;
             if (c < k) {
                 double sq = 0.0;
@@ -387,7 +425,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
                 c2 = (float)sq;
             }
             const float q1 = bfr(c2), q2 = bfr(__fsub_rn(c2, q1)), q3 = bfr(__fsub_rn(__fsub_rn(c2, q1), q2));
-            v = j == d ? q1 : (j == d + 1 ? q2 : q3);
+            v = aug == 0 ? q1 : (aug == 1 ? q2 : q3);
         }
         *reinterpret_cast<__nv_bfloat16 *>(b1 + (nn >> 3) * SB1 + (kk >> 3) * 128 + (nn & 7) * 16 + (kk & 7) * 2) =
             __float2bfloat16_rn(v);
@@ -439,9 +477,9 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             KM_TRACE(s, 1);
             float nrm;
             if (full)
-                nrm = km_convert_row<true, EVEN>(src, d, true, G, qd, ta, xr, skip);
+                nrm = km_convert_row<true, EVEN, PKD>(src, d, true, G, qd, ta, xr, skip);
             else
-                nrm = km_convert_row<false, EVEN>(src, d, valid, G, qd, ta, xr, skip);
+                nrm = km_convert_row<false, EVEN, PKD>(src, d, valid, G, qd, ta, xr, skip);
             B.nrm[sa][r] = nrm;
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
             fence_proxy_async();
@@ -584,7 +622,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         constexpr uint32_t id2 = umma_idesc_bf16(NC, 1, 0);  // A (X) MN-major, B (one-hot) K-major
         if (warp == kKmWarpMma && lane == 0) {
             const uint32_t b10 = km_smem(b1);
-            const int K1S = 2 * G.KP / 16;  // MMA1 instructions (K = 16 each)
+            const int K1S = K1 / 16;  // MMA1 instructions (K = 16 each)
             const uint64_t bdesc0 = umma_desc(b10, 128, SB1);
             for (int s1 = 0; s1 < ns; ++s1) {
                 const int sa = s1 % kKmNA;
