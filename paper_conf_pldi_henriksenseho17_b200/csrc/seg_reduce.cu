@@ -88,6 +88,69 @@ seg_tile_kernel(const T *__restrict__ x, int64_t nseg, int L, int tile_segs, T *
     }
 }
 
+
+// ---------------------------------------------------------------- KG1b (odd L <= 64)
+// Short rows of odd length: tiles of R = 256 k whole rows (R L elements, <= ~32 KB) stream into a
+// 2-slot shared-memory ring by 1-D TMA bulk copies (the next tile lands while this one is
+// reduced), then thread t folds rows t, t + 256, ... in index order.  A row is L consecutive
+// words: an odd stride, so the 32 lanes' loads fall in 32 distinct banks.  No padding, no
+// staging instructions, one coalesced output store per row.
+constexpr int kRowsTileElems = 8192;
+__host__ __device__ inline int rows_tile_rows(int L) {
+    const int k = kRowsTileElems / (256 * L);
+    return 256 * (k > 1 ? k : 1);
+}
+template <int OP, typename T>
+__global__ void __launch_bounds__(256)
+seg_rows_odd_kernel(const T *__restrict__ x, int64_t nseg, int L, T *out, int64_t *out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bars[2];
+    const int t = threadIdx.x;
+    const int R = rows_tile_rows(L);
+    const int64_t ntiles = (nseg + R - 1) / R, nfull = nseg / R;
+    const unsigned tile_bytes = (unsigned)(R * L * (int)sizeof(T));
+    T *slot[2] = {reinterpret_cast<T *>(smem_raw), reinterpret_cast<T *>(smem_raw + tile_bytes)};
+    if (t == 0) {
+        mbar_init(&bars[0], 1);
+        mbar_init(&bars[1], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    // tiles b, b + G, ...: the i-th of this CTA uses slot i & 1, phase (i >> 1) & 1
+    auto issue = [&](int64_t tile, int sl) {
+        if (tile < nfull) {
+            mbar_expect_tx(&bars[sl], tile_bytes);
+            tma_load_1d(slot[sl], x + tile * R * (int64_t)L, tile_bytes, &bars[sl]);
+        }
+    };
+    if (t == 0) {
+        issue(blockIdx.x, 0);
+        issue(blockIdx.x + gridDim.x, 1);
+    }
+    int i = 0;
+    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++i) {
+        const int sl = i & 1;
+        const int64_t r0 = tile * R;
+        const int rows = (int)(nseg - r0 < R ? nseg - r0 : R);
+        const bool full = tile < nfull;
+        if (full) mbar_wait(&bars[sl], (unsigned)((i >> 1) & 1));
+        const T *src = full ? slot[sl] : x + r0 * (int64_t)L;  // the ragged last tile from global memory
+        for (int r = t; r < rows; r += 256) {
+            const T *row = src + (int64_t)r * L;
+            V a = O::id();
+            for (int j = 0; j < L; ++j) a = O::fold(a, row[j], j);
+            store_out<O>(out, out_idx, r0 + r, a);
+        }
+        __syncthreads();  // every thread is done with the slot before it is refilled
+        if (t == 0) {
+            fence_proxy_async();
+            issue(tile + 2 * (int64_t)gridDim.x, sl);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- KG0
 // Power-of-two segments up to 32 vectors, 16-byte aligned base: no shared
 // memory at all.  Each lane loads 16-byte vectors straight from HBM (coalesced,
@@ -426,6 +489,19 @@ template <int OP, typename T> struct SegRun {
             grid = grid < cap ? grid : cap;
             seg_vec_kernel<OP, T, kSegThreads, 4><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, G,
                                                                                          (T *)out, out_idx);
+            return launch_status();
+        }
+        if (regime == 0 && (L & 1) && L <= 64 && ((uintptr_t)x & 15) == 0 &&
+            2 * rows_tile_rows((int)L) * L * (int64_t)sizeof(T) <= 160 * 1024) {
+            const int R = rows_tile_rows((int)L);
+            const int smem = 2 * R * (int)L * (int)sizeof(T);
+            auto kr = seg_rows_odd_kernel<OP, T>;
+            if (smem > 32 * 1024)
+                cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+            const int64_t ntiles = ceil_div(nseg, R);
+            const int64_t cap = resident_blocks((const void *)kr, 256, (size_t)smem);
+            const int64_t grid = ntiles < cap ? ntiles : cap;
+            kr<<<(unsigned)(grid > 0 ? grid : 1), 256, smem, st>>>(x, nseg, (int)L, (T *)out, out_idx);
             return launch_status();
         }
         if (regime == 0) {

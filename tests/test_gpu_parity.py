@@ -425,6 +425,28 @@ def test_seg_reduce_col_major(fs, dt, op, nseg, seglen):
             np.testing.assert_array_equal(host(row), host(got))
 
 
+@pytest.mark.parametrize("dt", DTYPES)
+@pytest.mark.parametrize("op", OPS)
+@pytest.mark.parametrize("nseg,seglen,layout", [
+    (3 * 2560 + 17, 3, "row"), (8192 * 2 + 5, 1, "row"), (1001, 33, "row"), (777, 63, "row"), (2049, 31, "row"),
+    (310_001, 3, "col"), (303_105, 7, "col"), (256, 100_003, "col"), (5, 200_003, "col"), (64, 400_009, "col"),
+    (268, 5_003, "col"), (1024, 4_099, "col"), (1000, 4_096, "col"), (3, 9_001, "col"), (1, 70_001, "col"),
+    (1025, 5_000, "col")])
+def test_seg_reduce_tiled_rows_and_split_columns(fs, dt, op, nseg, seglen, layout):
+    """Row layout, odd seglen <= 63: whole rows staged by TMA, one thread per row, several tiles
+    and a ragged last tile.  Column layout: m <= 8 rows of >= 148*8*256 columns (the short-rows
+    kernel), narrow w <= 1024 read as one flat vector stream (periods of rows, leftover rows), and
+    hundreds of row splits (the two-level combine of partial rows)."""
+    x = workloads.mixed(nseg * seglen, nseg ^ seglen, dt)
+    got = fs.seg_reduce(cu(x), nseg, seglen, op, layout=layout)
+    want = oracle.seg_reduce(x, nseg, seglen, op, layout)
+    asum = oracle.seg_reduce(np.abs(x), nseg, seglen, "add", layout) if (op == "add" and dt == np.float32) else None
+    assert_reduced(got, want, op, asum, f"{layout} {nseg}x{seglen}")
+    if layout == "col" and nseg * seglen < (1 << 22):  # misaligned base: the short-rows kernel takes any phase
+        got = fs.seg_reduce(cu(x, 1), nseg, seglen, op, layout=layout)
+        assert_reduced(got, want, op, asum, f"{layout} {nseg}x{seglen} misaligned")
+
+
 def test_seg_reduce_empty(fs):
     for op in OPS:
         got = fs.seg_reduce(torch.zeros(0, dtype=torch.float32, device="cuda"), 5, 0, op)

@@ -104,5 +104,18 @@ fs.argmin_unpack(k8, torch.int64, P=9)
 pk = fs.partials_pack(cu(workloads.mixed((5, 7), 14, np.float32)), cu(np.arange(5, dtype=np.int32)))
 fs.partials_unpack(pk, torch.empty((5, 7), device="cuda"), torch.empty(5, dtype=torch.int32, device="cuda"))
 fs.copy_2d(x[1:], 33, 17, 41, torch.empty(33 * 19 + 1, device="cuda")[1:], 19)
+# seg_reduce: odd short rows staged by TMA (several tiles + ragged tail), column layout short
+# rows (m <= 8, >= 148*8*256 columns), the flat period stream (w <= 1024) and two-level split combine
+xs = cu(workloads.mixed(2_200_000, 15, np.float32))
+xs8 = cu(workloads.mixed(2_200_000, 16, np.int64))
+for nseg, L in ((7697, 3), (1001, 33), (777, 63), (2049, 31)):
+    fs.seg_reduce(xs[: nseg * L], nseg, L, "add")
+    fs.seg_reduce(xs8[: nseg * L], nseg, L, "argmin")
+fs.seg_reduce(xs[: 310_001 * 7], 310_001, 7, "argmin", layout="col")
+fs.seg_reduce(xs[1: 1 + 310_001 * 3], 310_001, 3, "add", layout="col")
+for nseg, L in ((268, 5_003), (3, 9_001), (512, 4_099), (5, 200_003), (64, 30_001)):
+    fs.seg_reduce(xs[: nseg * L], nseg, L, "add", layout="col")
+    fs.seg_reduce(xs8[: nseg * L], nseg, L, "argmin", layout="col")
+    fs.seg_reduce(xs[1: 1 + nseg * L], nseg, L, "max", layout="col")
 torch.cuda.synchronize()
 print("sanitize cases done")

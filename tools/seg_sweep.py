@@ -35,18 +35,25 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--auto-only", action="store_true", help="skip the forced-regime rows")
+    ap.add_argument("--seglens", default="", help="comma-separated subset of C4 seglens")
+    ap.add_argument("--what", default="reduce,scan", help="reduce and/or scan")
     args = ap.parse_args()
     n = 1 << (24 if args.quick else 28)
     x = workloads.device_uniform(n, 5, "cuda")
     rows = []
     seglens = [L for L in workloads.C4_SEGLENS if L <= n]
+    if args.seglens:
+        keep = {int(v) for v in args.seglens.split(",")}
+        seglens = [L for L in seglens if L in keep]
+    what = set(args.what.split(","))
     for L in seglens:
         nseg = n // L
         m = nseg * L
         xv = x[:m]
         red_bytes = 4 * m + 4 * nseg
         rec = {"seglen": L, "nseg": nseg, "auto_regime": fs.seg_regime(nseg, L)}
-        for reg in (-1, 0, 1, 2, 3):
+        for reg in ((-1,) if args.auto_only else (-1, 0, 1, 2, 3)) if "reduce" in what else ():
             if reg == 0 and L > 8192:
                 continue
             if reg in (1,) and L > (1 << 22):
@@ -58,9 +65,14 @@ def main():
             finally:
                 fs.force_seg_regime(-1)
             rec[f"reduce_row_r{reg}_GBs"] = round(red_bytes / ms / 1e6, 1)
-        out = torch.empty(nseg, device="cuda")
-        ms = timeit(lambda: fs.seg_reduce(xv, nseg, L, "add", layout="col", out=out), args.reps)
-        rec["reduce_col_GBs"] = round(red_bytes / ms / 1e6, 1)
+        if "reduce" in what:
+            out = torch.empty(nseg, device="cuda")
+            ms = timeit(lambda: fs.seg_reduce(xv, nseg, L, "add", layout="col", out=out), args.reps)
+            rec["reduce_col_GBs"] = round(red_bytes / ms / 1e6, 1)
+        if "scan" not in what:
+            rows.append(rec)
+            print(json.dumps(rec), file=sys.stderr, flush=True)
+            continue
         sout = torch.empty(m, device="cuda")
         ms = timeit(lambda: fs.seg_scan(xv, nseg, L, "add", out=sout), args.reps)
         rec["scan_row_GBs"] = round(8 * m / ms / 1e6, 1)
