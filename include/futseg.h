@@ -327,7 +327,8 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       512 i64), 16-byte aligned buffers: in-register + shuffle scan, a shared-memory
  *       combine across the warps of a CTA for rows longer than 32 vectors
  *   8 = KS1 rows of 2..32 elements that are not powers of two, op != ARGMIN, 16-byte
- *       aligned: 256 rows staged through shared memory, a thread scans a row
+ *       aligned input when the output is not (else KS3 takes them): 256 rows staged
+ *       through shared memory, a thread scans a row
  *   9 = KS2 rows of >= 4 chunks of 256 x R vectors (12288 f32/i32 add/min/max, 4096
  *       argmin, 2048 i64) when there are at least as many rows as SMs (in/out with the
  *       same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with a
@@ -335,9 +336,12 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *  10 = KS0-BIG power-of-two rows of 2-8 CTA steps (256 < seglen/VEC <= 2048: 2048..8192
  *       f32/i32, 1024..4096 i64), 16-byte aligned: a CTA loads a whole row per step,
  *       warp 0 scans the warp totals
- *  11 = KS3 rows of 32 < seglen <= 16384 (8192 for i64), op != ARGMIN, element-aligned:
- *       R whole rows per CTA staged in shared memory, odd-length per-thread pieces, a
- *       CTA scan of the piece summaries (no look-back)
+ *  11 = KS3 rows of 32 < seglen <= 16384 (8192 for i64), op != ARGMIN, element-aligned,
+ *       and rows of 2..32 elements (not powers of two) with 16-byte aligned input and
+ *       output: R whole rows per CTA staged in shared memory (by TMA bulk copies through
+ *       a 3-slot ring and TMA bulk stores when both buffers are 16-byte aligned and a tile
+ *       of R rows is <= 72 KB), odd-length per-thread pieces, a CTA scan of the piece
+ *       summaries (no look-back)
  *  12 = flat (unsegmented) slab scan per row: one row (nseg == 1), or fewer rows than SMs
  *       of >= 2^26 elements each, 16-byte aligned
  * fs_seg_regime returns the regime a call with these sizes takes on the current device

@@ -46,7 +46,7 @@ REGIMES = {0: "KG0/KG1 short rows (shuffle groups / smem tile)", 1: "KG2 warp/se
            3: "KG4 multi-block/segment", 4: "column (col-major)", 5: "segmented look-back scan", 6: "empty",
            7: "KS0 short power-of-two scan (register + shuffle)", 8: "KS1 short-row scan (shared-memory tile)",
            9: "KS2 CTA-per-row scan with a running carry", 10: "KS0-BIG power-of-two rows of 2-8 CTA steps",
-           11: "KS3 whole rows staged in shared memory", 12: "flat slab scan per row"}
+           11: "KS3 whole rows staged in shared memory (TMA ring when aligned)", 12: "flat slab scan per row"}
 
 
 class fs_opdesc(ctypes.Structure):

@@ -1105,6 +1105,116 @@ segscan_rows_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, int64_t R,
     }
 }
 
+// KS3 with TMA (16-byte aligned input and output): the same piece scan, but tiles of R whole
+// rows (R * L * sizeof(T) a multiple of 16 bytes, <= 72 KB) arrive by TMA bulk copies into a
+// 3-slot ring (the tile two ahead is in flight while this one is scanned) and leave by TMA bulk
+// stores straight from shared memory; one CTA loop per resident slot.  Full tiles only: the
+// nseg mod R leftover rows take segscan_rows_kernel.
+template <int OP, typename T>
+__global__ void __launch_bounds__(256)
+segscan_rows_tma_kernel(const T *__restrict__ x, int64_t ntiles, int64_t L, int R, T *__restrict__ out) {
+    using O = Op<OP, T>;
+    extern __shared__ __align__(128) unsigned char smem_rt[];
+    __shared__ uint64_t full[3];
+    __shared__ T s_wa[8];
+    __shared__ int s_wf[8];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int cnt = (int)(R * L);
+    const unsigned TB = (unsigned)cnt * sizeof(T);
+    const int64_t G = gridDim.x;
+    const int my = (int)((ntiles - blockIdx.x + G - 1) / G);
+    auto issue = [&](int i) {  // thread 0: load this CTA's i-th tile into slot i % 3
+        const int64_t tile = blockIdx.x + (int64_t)i * G;
+        mbar_expect_tx(&full[i % 3], TB);
+        tma_load_1d(smem_rt + (i % 3) * TB, x + tile * cnt, TB, &full[i % 3]);
+    };
+    if (tid == 0) {
+        for (int q = 0; q < 3; ++q) mbar_init(&full[q], 1);
+        fence_mbar_init();
+        for (int i = 0; i < 2 && i < my; ++i) issue(i);
+    }
+    __syncthreads();
+    const int E = ((cnt + 255) / 256) | 1;  // odd piece length: the lanes' strided reads hit distinct banks
+    const int i0 = tid * E < cnt ? tid * E : cnt, i1 = i0 + E < cnt ? i0 + E : cnt;
+    const int jstart = (int)(i0 % L);
+    for (int it = 0; it < my; ++it) {
+        const int64_t tile = blockIdx.x + (int64_t)it * G;
+        T *buf = reinterpret_cast<T *>(smem_rt + (it % 3) * TB);
+        mbar_wait(&full[it % 3], (unsigned)(it / 3) & 1u);
+        int j = jstart;
+        T acc = O::id();
+        int f = 0;
+        for (int i = i0; i < i1; ++i) {
+            const T v = buf[i];
+            if (j == 0) {
+                acc = v;
+                f = 1;
+            } else {
+                acc = O::comb(acc, v);
+            }
+            buf[i] = acc;
+            if (++j == L) j = 0;
+        }
+        T a = acc;
+        int fl = f;
+#pragma unroll
+        for (int dd = 1; dd < 32; dd <<= 1) {
+            const T ya = shfl_up(a, dd);
+            const int yf = __shfl_up_sync(0xffffffffu, fl, dd);
+            if (lane >= dd) {
+                if (!fl) a = O::comb(ya, a);
+                fl |= yf;
+            }
+        }
+        if (lane == 31) {
+            s_wa[warp] = a;
+            s_wf[warp] = fl;
+        }
+        __syncthreads();
+        T ex = shfl_up(a, 1);
+        int exf = __shfl_up_sync(0xffffffffu, fl, 1);
+        if (lane == 0) {
+            ex = O::id();
+            exf = 0;
+        }
+        if (!exf) {
+            T p = O::id();
+            for (int q = 0; q < warp; ++q) p = s_wf[q] ? s_wa[q] : O::comb(p, s_wa[q]);
+            ex = O::comb(p, ex);
+        }
+        {
+            int jj = jstart;
+            for (int i = i0; i < i1 && jj != 0; ++i) {
+                buf[i] = O::comb(ex, buf[i]);
+                if (++jj == L) jj = 0;
+            }
+        }
+        fence_proxy_async();  // generic-proxy writes -> visible to the bulk store
+        __syncthreads();
+        if (tid == 0) {
+            tma_store_1d(out + tile * cnt, buf, TB);
+            bulk_commit();
+            if (it + 2 < my) {
+                if (it >= 1) bulk_wait_read<1>();  // the store of slot (it + 2) % 3 (iteration it - 1) has read it
+                issue(it + 2);
+            }
+        }
+    }
+    if (tid == 0) bulk_wait_read<0>();
+}
+
+// rows per tile of the TMA KS3 path (R * L * es a multiple of 16 bytes, <= 72 KB), 0 if none
+static int64_t ks3_tma_rows(int64_t L, int64_t es) {
+    const int64_t VEC = 16 / es;
+    int64_t g = VEC;  // gcd(L, VEC), VEC a power of two
+    while (L % g) g >>= 1;
+    const int64_t step = VEC / g;  // rows whose elements fill whole 16-byte vectors
+    int64_t R = (kRowsElems / L) / step * step;
+    if (R < step) R = step;
+    if (R * L * es > 72 * 1024) return 0;  // 3 slots <= 216 KB
+    return R;
+}
+
 // KS1: short rows of any length L <= 32 that are not powers of two (a 16-byte vector then
 // straddles rows): a CTA stages 256 whole rows through shared memory with coalesced 16-byte
 // loads (index padded every 32 elements), thread t scans row t sequentially in place, and
@@ -1314,7 +1424,8 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
         op != FS_ARGMIN && al16 && plain && L >= 2 && L <= 32,                        // 8 KS1
         plain && co16 && elem && L >= 4 * ks2ch && nseg_ok(n, L),                     // 9 KS2
         al16 && plain && pow2 && L > 256 * VEC && L <= 2048 * VEC,                    // 10 KS0-BIG
-        op != FS_ARGMIN && plain && elem && L > 32 && L <= (es == 4 ? 16384 : 8192),  // 11 KS3
+        op != FS_ARGMIN && plain && elem && L <= (es == 4 ? 16384 : 8192) &&          // 11 KS3
+            (L > 32 || (L >= 2 && al16 && ks3_tma_rows(L, es) > 0)),
         al16 && plain && (L * es) % 16 == 0,                                          // 12 flat per row
     };
     const int f = forced_seg_regime();
@@ -1433,6 +1544,28 @@ template <int OP, typename T> struct ScanRun {
                 return launch_status();
             }
             if constexpr (OP != kArgmin) {  // (argmin's index output keeps the look-back path)
+                if (rg == RG_KS3 && al && ks3_tma_rows(L, sizeof(T)) > 0 && n / L >= ks3_tma_rows(L, sizeof(T))) {
+                    const int64_t R = ks3_tma_rows(L, sizeof(T)), nseg = n / L, ntiles = nseg / R;
+                    auto kt = segscan_rows_tma_kernel<OP, T>;
+                    const int smem = (int)(3 * R * L * (int64_t)sizeof(T));
+                    cudaFuncSetAttribute((const void *)kt, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                    int64_t grid = resident_blocks((const void *)kt, 256, (size_t)smem);
+                    grid = grid > ntiles ? ntiles : grid;
+                    kt<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, ntiles, L, (int)R, (T *)out);
+                    const int64_t done = ntiles * R;
+                    if (done < nseg) {  // leftover rows: the staged-load KS3
+                        auto kr = segscan_rows_kernel<OP, T>;
+                        const int64_t R2 = L >= kRowsElems ? 1 : kRowsElems / L;
+                        const int sm2 = (int)(R2 * L * (int64_t)sizeof(T));
+                        if (sm2 > 32 * 1024)
+                            cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, sm2);
+                        const int64_t g2 = ceil_div(nseg - done, R2);
+                        kr<<<(unsigned)g2, 256, sm2, st>>>((const T *)in0 + done * L, nseg - done, L, R2,
+                                                          (T *)out + done * L);
+                        return launch_status(2);
+                    }
+                    return launch_status();
+                }
                 if (rg == RG_KS3) {
                     auto kr = segscan_rows_kernel<OP, T>;
                     const int64_t nseg = n / L;

@@ -209,7 +209,7 @@ def test_workspace_queries_and_regimes(fs):
     assert r(4, 1 << 26) == 3 and r(1, 1 << 28) == 3
     assert r(64, 64, layout="col") == 4
     assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 11
-    assert r(1 << 20, 3, scan=True) == 8 and r(1 << 20, 33, scan=True) == 11 and r(64, 7, scan=True, op="argmin") == 5
+    assert r(1 << 20, 3, scan=True) == 11 and r(1 << 20, 33, scan=True) == 11 and r(64, 7, scan=True, op="argmin") == 5
     assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 11  # KS2: >= 1 row per SM
     assert r(64, 16384, scan=True, op="argmin") == 5 and r(64, 16385, scan=True) == 5
     assert r(1 << 12, 2048, scan=True) == 10 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 10
@@ -226,7 +226,7 @@ def test_workspace_queries_and_regimes(fs):
         fs.force_seg_regime(-1)
     assert r(1 << 20, 16) == 0
     for forced, shape, want in ((5, (1 << 20, 1024), 5), (12, (1 << 10, 1024), 12), (11, (1 << 10, 1024), 11),
-                                (12, (1 << 20, 3), 8), (11, (64, 63), 11), (9, (1 << 12, 2048), 10)):
+                                (12, (1 << 20, 3), 11), (8, (1 << 20, 3), 8), (11, (64, 63), 11), (9, (1 << 12, 2048), 10)):
         fs.force_seg_regime(forced)
         try:
             assert r(*shape, scan=True) == want, (forced, shape)

@@ -496,8 +496,9 @@ def test_seg_scan_short_pow2(fs, nseg, seglen):
 @pytest.mark.parametrize("nseg,seglen", [(4, 70_001), (8, 4096), (16, 100_003), (32, 9_999), (2, 300_007),
                                          (4, 2_000_000)])
 def test_seg_scan_col_narrow(fs, nseg, seglen):
-    """Column-major seg_scan with few columns (rows of <= 8 16-byte vectors): the warp-per-
-    row-block kernels (partial, carry, scan); ragged row blocks; argmin ties; 8-byte types."""
+    """Column-major seg_scan with few columns (rows of <= 8 16-byte vectors): the one-pass
+    look-back kernel (blocks stacked down the columns, per-column look-back); ragged row
+    blocks; argmin ties; 8-byte types."""
     for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
                    (np.int64, "add"), (np.int32, "max")):
         if np.dtype(dt).itemsize == 8 and nseg > 16:
@@ -515,8 +516,9 @@ def test_seg_scan_col_narrow(fs, nseg, seglen):
                                          (128 * 37, 777), (1 << 17, 64)])
 def test_seg_scan_col_wide(fs, nseg, seglen):
     """Column-major seg_scan with wide rows (multiples of 128 four-byte columns, 16-byte
-    vectors): the three-pass kernels (partials, carries, scan) with ragged row blocks,
-    int wrap-around, 8-byte types and argmin."""
+    vectors): the one-pass look-back kernel over several column tiles (or one thread per
+    column when no row split is needed) with ragged row blocks, int wrap-around, 8-byte
+    types and argmin."""
     for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int32, "min"), (np.float32, "max"),
                    (np.float32, "min"), (np.int64, "add"), (np.float32, "argmin")):
         x = workloads.mixed(nseg * seglen, nseg * 5 + seglen, dt)
@@ -526,6 +528,23 @@ def test_seg_scan_col_wide(fs, nseg, seglen):
         want = oracle.seg_scan(x, nseg, seglen, op, "col")
         asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", "col") if (op == "add" and dt == np.float32) else None
         assert_reduced(got, want, op, asum, f"segscan col wide {nseg}x{seglen} {dt.__name__} {op}")
+
+
+@pytest.mark.parametrize("nseg,seglen,offset", [(303_105, 3, 0), (310_001, 7, 1), (303_104, 2, 0), (5, 100_003, 0),
+                                                (37, 20_011, 0), (3, 1_000_003, 0), (200, 5_000, 1), (33, 40_000, 2)])
+def test_seg_scan_col_short_and_scalar(fs, nseg, seglen, offset):
+    """Column layout: m <= 8 rows of >= 148 * 2048 columns (the short-rows kernel, any phase),
+    and widths that are not multiples of the vector (or misaligned views): scalar columns
+    through the one-pass look-back kernel."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.float32, "argmin"), (np.int64, "min"),
+                   (np.int32, "max")):
+        x = workloads.mixed(nseg * seglen, nseg * 11 + seglen, dt)
+        if op == "argmin":
+            x[::4] = x.min()
+        got = fs.seg_scan(cu(x, offset), nseg, seglen, op, layout="col")
+        want = oracle.seg_scan(x, nseg, seglen, op, "col")
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", "col") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan col {nseg}x{seglen}+{offset} {dt.__name__} {op}")
 
 
 def test_seg_scan_few_long_rows(fs):
@@ -560,16 +579,27 @@ def test_seg_scan_pow2_misaligned_falls_back(fs, seglen):
 
 @pytest.mark.parametrize("seglen", [3, 5, 7, 9, 12, 17, 31])
 @pytest.mark.parametrize("nseg", [1, 2, 255, 256, 257, 100_001])
-def test_seg_scan_short_rows_tile(fs, nseg, seglen):
-    """KS1 (regime 8): short non-power-of-two rows staged through shared memory (tiles of 256
-    rows, a ragged last tile, scalar tails of the vector loads); add/min/max on every dtype."""
-    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int32, "max"), (np.int64, "add")):
-        x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
-            workloads.mixed(nseg * seglen, nseg + seglen, dt)
-        got = fs.seg_scan(cu(x), nseg, seglen, op)
-        want = oracle.seg_scan(x, nseg, seglen, op)
-        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
-        assert_reduced(got, want, op, asum, f"segscan tile {nseg}x{seglen} {dt.__name__} {op}")
+@pytest.mark.parametrize("regime", [-1, 8])
+def test_seg_scan_short_rows_tile(fs, nseg, seglen, regime):
+    """Short non-power-of-two rows: KS3 with the TMA ring (regime 11, the default for aligned
+    buffers: tiles of R rows, R a multiple of the rows that fill whole 16-byte vectors, the
+    leftover rows by the staged-load KS3) and KS1 forced (regime 8: tiles of 256 rows, a ragged
+    last tile, scalar tails of the vector loads); add/min/max on every dtype."""
+    fs.force_seg_regime(regime)
+    try:
+        for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int32, "max"),
+                       (np.int64, "add")):
+            x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
+                workloads.mixed(nseg * seglen, nseg + seglen, dt)
+            got = fs.seg_scan(cu(x), nseg, seglen, op)
+            if nseg > 1:
+                want_rg = 8 if regime == 8 else 11
+                assert fs.last_seg_regime() == want_rg, (fs.last_seg_regime(), want_rg)
+            want = oracle.seg_scan(x, nseg, seglen, op)
+            asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+            assert_reduced(got, want, op, asum, f"segscan tile {nseg}x{seglen} {dt.__name__} {op} r={regime}")
+    finally:
+        fs.force_seg_regime(-1)
 
 
 @pytest.mark.parametrize("seglen", [33, 100, 1000, 1023, 4097, 8191, 9000, 16_383])

@@ -117,5 +117,17 @@ for nseg, L in ((268, 5_003), (3, 9_001), (512, 4_099), (5, 200_003), (64, 30_00
     fs.seg_reduce(xs[: nseg * L], nseg, L, "add", layout="col")
     fs.seg_reduce(xs8[: nseg * L], nseg, L, "argmin", layout="col")
     fs.seg_reduce(xs[1: 1 + nseg * L], nseg, L, "max", layout="col")
+# seg_scan column layout: the one-pass look-back kernel (vector / scalar columns, 8-byte, argmin)
+# and the short-rows kernel
+for nseg, L in ((512, 2_049), (5, 30_001), (2, 100_003), (4096, 65)):
+    fs.seg_scan(xs[: nseg * L], nseg, L, "add", layout="col")
+    fs.seg_scan(xs8[: nseg * L], nseg, L, "argmin", layout="col")
+    fs.seg_scan(xs[1: 1 + nseg * L], nseg, L, "max", layout="col")
+fs.seg_scan(xs[1: 1 + 303_105 * 3], 303_105, 3, "add", layout="col")
+fs.seg_scan(xs[: 303_105 * 7], 303_105, 7, "argmin", layout="col")
+# seg_scan KS3 through the TMA ring (short and long rows, 8-byte, leftover rows)
+for nseg, L in ((30_001, 3), (9_001, 7), (1_001, 33), (77, 1000), (50, 4097)):
+    fs.seg_scan(xs[: nseg * L], nseg, L, "add")
+    fs.seg_scan(xs8[: nseg * L], nseg, L, "max")
 torch.cuda.synchronize()
 print("sanitize cases done")

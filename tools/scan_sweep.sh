@@ -13,7 +13,8 @@ if [ "$1" = build ]; then
   objs=$(ls $ROOT/paper_conf_pldi_henriksenseho17_b200/_build/*.o | grep -v '/scan.o')
   for v in $VARIANTS; do
     flags=""
-    for kv in ${v//_/ }; do k=$(echo $kv | sed 's/[0-9]*$//'); val=${kv#$k}; flags="$flags -DFS_SCANW_$k=$val"; done
+    for kv in ${v//_/ }; do k=$(echo $kv | sed 's/[0-9]*$//'); val=${kv#$k}
+      case $k in X*) flags="$flags -DFS_SCANR_${k#X}=$val";; I*) flags="$flags -DFS_SCAN_IMPL=$val";; *) flags="$flags -DFS_SCANW_$k=$val";; esac; done
     ( nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 --expt-relaxed-constexpr -I$ROOT/include -I$CS $flags \
         -c $CS/scan.cu -o $OUT/scan_$v.o && \
       nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -I$ROOT/include $ROOT/tools/scan_sweep.cu \
