@@ -766,7 +766,15 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
             };
             auto seg_idx = [&](int i) -> int64_t { return i < i0 ? r0 + i : i - i0; };  // one-start case
             S tot = SO::id();
-            if (one) {
+            // fast path (a full tile, no segment start among this thread's elements): a plain
+            // fold, no per-element validity or restart tests
+            const bool plainrun = full && (!SEG || (one && i0 >= E));
+            if (plainrun) {
+                V acc = O::id();
+#pragma unroll
+                for (int i = 0; i < E; ++i) acc = O::comb(acc, O::lift(x[i], SEG ? r0 + i : ibase + e0 + i));
+                tot = S{acc, 0};
+            } else if (one) {
                 V acc = O::id();
 #pragma unroll
                 for (int i = 0; i < E; ++i)
@@ -802,7 +810,15 @@ scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T 
             S run = SO::comb(run_c, SO::comb(wex, tex));
             run_c = SO::comb(run_c, tagg);
             T y[E];
-            if (one) {
+            if (plainrun) {
+                V acc = run.v;
+#pragma unroll
+                for (int i = 0; i < E; ++i) {
+                    acc = O::comb(acc, O::lift(x[i], SEG ? r0 + i : ibase + e0 + i));
+                    y[i] = O::val(acc);
+                    if (OP == kArgmin) out_idx[e0 + i] = O::idx(acc);
+                }
+            } else if (one) {
                 V acc = run.v;
 #pragma unroll
                 for (int i = 0; i < E; ++i) {
@@ -1203,6 +1219,91 @@ segscan_rows_tma_kernel(const T *__restrict__ x, int64_t ntiles, int64_t L, int 
     if (tid == 0) bulk_wait_read<0>();
 }
 
+// KS2 with TMA (16-byte aligned buffers, seglen a multiple of the vector width): a CTA owns
+// whole rows (rows b, b + G, ...) and streams each row through a 3-slot TMA ring in tiles of up
+// to kRowStreamElems elements (the tile two ahead in flight), scans the tile in shared memory
+// (odd-length thread pieces, a CTA scan of the piece totals, the row's running carry) and
+// stores it with a TMA bulk store.  No look-back; every element crosses HBM once each way.
+constexpr int kRowStreamElems = 8192;
+template <int OP, typename T>
+__global__ void __launch_bounds__(256)
+segscan_rowstream_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restrict__ out) {
+    using O = Op<OP, T>;
+    extern __shared__ __align__(128) unsigned char smem_rs[];
+    __shared__ uint64_t full[3];
+    __shared__ T s_wa[8];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    constexpr int CH = kRowStreamElems;
+    constexpr unsigned SLOT = CH * sizeof(T);
+    const int64_t G = gridDim.x;
+    const int64_t nch = (L + CH - 1) / CH;  // tiles per row
+    const int64_t myrows = (nseg - blockIdx.x + G - 1) / G;
+    const int64_t my = myrows * nch;
+    auto item = [&](int64_t i, int64_t &row, int64_t &c) {
+        row = blockIdx.x + (i / nch) * G;
+        c = i % nch;
+    };
+    auto issue = [&](int64_t i) {  // thread 0: this CTA's i-th tile into slot i % 3
+        int64_t row, c;
+        item(i, row, c);
+        const int64_t cnt = L - c * CH < CH ? L - c * CH : CH;
+        mbar_expect_tx(&full[i % 3], (unsigned)(cnt * sizeof(T)));
+        tma_load_1d(smem_rs + (i % 3) * SLOT, x + row * L + c * CH, (unsigned)(cnt * sizeof(T)), &full[i % 3]);
+    };
+    if (tid == 0) {
+        for (int q = 0; q < 3; ++q) mbar_init(&full[q], 1);
+        fence_mbar_init();
+        for (int64_t i = 0; i < 2 && i < my; ++i) issue(i);
+    }
+    __syncthreads();
+    T carry = O::id();
+    for (int64_t it = 0; it < my; ++it) {
+        int64_t row, c;
+        item(it, row, c);
+        const int cnt = (int)(L - c * CH < CH ? L - c * CH : CH);
+        T *buf = reinterpret_cast<T *>(smem_rs + (it % 3) * SLOT);
+        if (c == 0) carry = O::id();
+        mbar_wait(&full[it % 3], (unsigned)(it / 3) & 1u);
+        const int E = ((cnt + 255) / 256) | 1;  // odd: the lanes' strided reads hit distinct banks
+        const int i0 = tid * E < cnt ? tid * E : cnt, i1 = i0 + E < cnt ? i0 + E : cnt;
+        T acc = O::id();
+        for (int i = i0; i < i1; ++i) {
+            acc = O::comb(acc, buf[i]);
+            buf[i] = acc;
+        }
+        T a = acc;  // inclusive warp scan of the piece totals
+#pragma unroll
+        for (int dd = 1; dd < 32; dd <<= 1) {
+            const T y = shfl_up(a, dd);
+            if (lane >= dd) a = O::comb(y, a);
+        }
+        if (lane == 31) s_wa[warp] = a;
+        __syncthreads();
+        T ex = shfl_up(a, 1);
+        if (lane == 0) ex = O::id();
+        T wp = carry, tot = carry;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            if (q < warp) wp = O::comb(wp, s_wa[q]);
+            tot = O::comb(tot, s_wa[q]);
+        }
+        const T base = O::comb(wp, ex);
+        for (int i = i0; i < i1; ++i) buf[i] = O::comb(base, buf[i]);
+        carry = tot;
+        fence_proxy_async();  // generic-proxy writes -> visible to the bulk store
+        __syncthreads();      // (also: s_wa is rewritten only after every thread has read it)
+        if (tid == 0) {
+            tma_store_1d(out + row * L + c * CH, buf, (unsigned)(cnt * sizeof(T)));
+            bulk_commit();
+            if (it + 2 < my) {
+                if (it >= 1) bulk_wait_read<1>();  // the store of slot (it + 2) % 3 has read it
+                issue(it + 2);
+            }
+        }
+    }
+    if (tid == 0) bulk_wait_read<0>();
+}
+
 // rows per tile of the TMA KS3 path (R * L * es a multiple of 16 bytes, <= 72 KB), 0 if none
 static int64_t ks3_tma_rows(int64_t L, int64_t es) {
     const int64_t VEC = 16 / es;
@@ -1395,7 +1496,10 @@ segscan_cta_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restri
 // KS2 applies when every SM gets at least one row: the rows are then the unit of parallelism
 // (seg sweep, profiles/r01_seg_sweep.json: at >= 1 row per SM KS2 beats the segmented look-back scan,
 // 256-268 rows 3.8 -> 4.8 TB/s, 512 rows 3.8 -> 4.5; below one row per SM SMs idle: 128 rows 3.6, 32 rows 1.1)
-static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm_count(); }
+#ifndef FS_KS2_MINF
+#define FS_KS2_MINF 85  // rows >= 0.85 x SMs: 128 rows of 2^21 0.736 (look-back) -> 0.751; 64 rows 0.41
+#endif
+static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm_count() * FS_KS2_MINF / 100; }
 #ifndef FS_FLAT_ROW_MIN
 #define FS_FLAT_ROW_MIN (1 << 26)
 #endif
@@ -1533,6 +1637,19 @@ template <int OP, typename T> struct ScanRun {
                 grid = grid > cap ? cap : (grid < 1 ? 1 : grid);
                 kb<<<(unsigned)grid, 256, 0, st>>>((const T *)in0, n, (int)L, (T *)out, out_idx);
                 return launch_status();
+            }
+            if constexpr (OP != kArgmin) {
+                if (rg == RG_KS2 && al && L % VEC == 0) {  // whole rows streamed through a TMA ring
+                    auto kr = segscan_rowstream_kernel<OP, T>;
+                    const int smem = 3 * kRowStreamElems * (int)sizeof(T);
+                    cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+                    const int64_t nseg = n / L;
+                    const int64_t cap = resident_blocks((const void *)kr, 256, (size_t)smem);
+                    const int64_t k = ceil_div(nseg, cap);  // rows per CTA, equal for all CTAs
+                    const int64_t grid = ceil_div(nseg, k);
+                    kr<<<(unsigned)grid, 256, smem, st>>>((const T *)in0, nseg, L, (T *)out);
+                    return launch_status();
+                }
             }
             if (rg == RG_KS2) {
                 constexpr int KS2R = ks2_rows<OP, T>();

@@ -619,6 +619,22 @@ def test_seg_scan_rows_ks3(fs, nseg, seglen, offset):
         assert_reduced(got, want, op, asum, f"segscan ks3 {nseg}x{seglen}+{offset} {dt.__name__} {op}")
 
 
+@pytest.mark.parametrize("nseg,seglen", [(149, 3 * 8192 + 4), (300, 20_000), (150, 65_536), (1000, 12_292)])
+def test_seg_scan_row_stream(fs, nseg, seglen):
+    """KS2 through the TMA ring (regime 9, 16-byte aligned, seglen a multiple of the vector):
+    rows of several 8192-element tiles and a partial last tile, equal rows per CTA; add/min/max
+    on every dtype, int wrap-around."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int64, "add"),
+                   (np.int32, "max"), (np.float32, "min")):
+        x = workloads.full_range(nseg * seglen, seglen, dt) if (op == "add" and dt != np.float32) else \
+            workloads.mixed(nseg * seglen, nseg + seglen, dt)
+        got = fs.seg_scan(cu(x), nseg, seglen, op)
+        assert fs.last_seg_regime() == 9, fs.last_seg_regime()
+        want = oracle.seg_scan(x, nseg, seglen, op)
+        asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add") if (op == "add" and dt == np.float32) else None
+        assert_reduced(got, want, op, asum, f"segscan stream {nseg}x{seglen} {dt.__name__} {op}")
+
+
 @pytest.mark.parametrize("seglen", [2048, 4097, 12_289, 16_384, 65_537])
 def test_seg_scan_cta_rows(fs, seglen):
     """KS2 (regime 9): a CTA owns whole rows (>= 4 rows per SM): whole and partial chunks,

@@ -129,5 +129,8 @@ fs.seg_scan(xs[: 303_105 * 7], 303_105, 7, "argmin", layout="col")
 for nseg, L in ((30_001, 3), (9_001, 7), (1_001, 33), (77, 1000), (50, 4097)):
     fs.seg_scan(xs[: nseg * L], nseg, L, "add")
     fs.seg_scan(xs8[: nseg * L], nseg, L, "max")
+# seg_scan KS2 through the TMA ring (rows of several tiles, partial last tile)
+fs.seg_scan(xs[: 149 * 12_292], 149, 12_292, "add")
+fs.seg_scan(xs8[: 150 * 12_292], 150, 12_292, "min")
 torch.cuda.synchronize()
 print("sanitize cases done")
