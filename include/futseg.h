@@ -327,8 +327,9 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       512 i64), 16-byte aligned buffers: in-register + shuffle scan, a shared-memory
  *       combine across the warps of a CTA for rows longer than 32 vectors
  *   8 = KS1 rows of 2..32 elements that are not powers of two, op != ARGMIN, 16-byte
- *       aligned input when the output is not (else KS3 takes them): 256 rows staged
- *       through shared memory, a thread scans a row
+ *       aligned: 256 rows staged through shared memory, a thread scans a row.  Taken only
+ *       when forced (fs_force_seg_regime): KS3's TMA ring is the plan's choice for these
+ *       rows since round 2 (L = 3: 0.57 -> 0.83 of the HBM roofline)
  *   9 = KS2 rows of >= 4 chunks of 256 x R vectors (12288 f32/i32 add/min/max, 4096
  *       argmin, 2048 i64) when there are at least as many rows as SMs (in/out with the
  *       same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with a

@@ -1980,11 +1980,172 @@ colscan_narrow_kernel(const T *__restrict__ x, int64_t m, int64_t w, int WV, int
     }
 }
 
+// ---------------------------------------------------------------- one-pass column-major seg_scan
+// Column-major seg_scan with row splitting in ONE pass (one read and one write per element): a
+// block is (column tile xt of CG vector-columns, row block y of RB thread-rows x K rows).  Each
+// CTA takes the next block id from an atomic counter (row-block-major, so the block above is
+// already owned by a running CTA), scans its K rows per thread in registers, combines the RB
+// thread-row totals of every column (Hillis-Steele over shared memory), and then -- one thread
+// per column -- runs a decoupled look-back up its column through the blocks above (published
+// per-(block, column) aggregate / inclusive prefix, TileState), i.e. F5 (L1071-1074) with the
+// chunks stacked down each column.  The three-kernel reduce / carry-scan / rescan above reads
+// every element twice (12 B per element).
+template <int OP, typename T, int VEC, int K>
+__global__ void __launch_bounds__(256)
+colscan_lb_kernel(const T *__restrict__ x, int64_t m, int64_t w, int CG, int64_t ntx, unsigned *counter,
+                  TileState<typename SOp<Op<OP, T>, false>::S, ScanShape<OP, T>::PACK> ts, T *__restrict__ out,
+                  int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    using SO = SOp<O, false>;
+    using S = typename SO::S;
+    constexpr int NT = 256;
+    __shared__ V sc[NT * VEC];
+    __shared__ V s_carry[NT];
+    __shared__ int64_t s_bid;
+    const int t = threadIdx.x;
+    const int RB = NT / CG, TCW = CG * VEC;
+    if (t == 0) s_bid = atomicAdd(counter, 1u);
+    __syncthreads();
+    const int64_t bid = s_bid;
+    const int64_t y = bid / ntx, xt = bid % ntx;
+    const int cg = t % CG, roff = t / CG;
+    const bool act = roff < RB;
+    const int64_t c = (xt * CG + cg) * VEC;
+    const bool colok = act && c < w;
+    const int64_t rbase = y * (int64_t)RB * K + (int64_t)roff * K;
+    V a[K][VEC];
+    if (VEC > 1) {
+        int4 raw[K];
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+            if (colok && rbase + j < m) raw[j] = ldg16(x + (rbase + j) * w + c);
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+            const Vec16<T> e = as_vec<T>(raw[j]);
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) a[j][k] = (colok && rbase + j < m) ? O::lift(e.e[k], rbase + j) : O::id();
+        }
+    } else {
+        T raw[K];
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+            if (colok && rbase + j < m) raw[j] = __ldg(x + (rbase + j) * w + c);
+#pragma unroll
+        for (int j = 0; j < K; ++j) a[j][0] = (colok && rbase + j < m) ? O::lift(raw[j], rbase + j) : O::id();
+    }
+#pragma unroll
+    for (int j = 1; j < K; ++j)
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) a[j][k] = O::comb(a[j - 1][k], a[j][k]);
+    if (act)
+#pragma unroll
+        for (int k = 0; k < VEC; ++k) sc[roff * TCW + cg * VEC + k] = a[K - 1][k];
+    __syncthreads();
+    for (int d = 1; d < RB; d <<= 1) {  // inclusive scan over the thread rows of every column
+        V v[VEC];
+        const bool up = act && roff >= d;
+        if (up)
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) v[k] = O::comb(sc[(roff - d) * TCW + cg * VEC + k], sc[roff * TCW + cg * VEC + k]);
+        __syncthreads();
+        if (up)
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) sc[roff * TCW + cg * VEC + k] = v[k];
+        __syncthreads();
+    }
+    if (t < TCW) {  // decoupled look-back up column t of the tile
+        const S agg{sc[(RB - 1) * TCW + t], 0};
+        S run = SO::id();
+        if (y == 0) {
+            ts.publish(bid * TCW + t, agg, kStIncl);
+        } else {
+            ts.publish(bid * TCW + t, agg, kStAgg);
+            int64_t p = bid - ntx;
+            while (true) {
+                S s;
+                const unsigned st = ts.poll(p * TCW + t, s);
+                if (st == 0) continue;
+                run = SO::comb(s, run);
+                if (st == kStIncl) break;
+                p -= ntx;
+            }
+            ts.publish(bid * TCW + t, SO::comb(run, agg), kStIncl);
+        }
+        s_carry[t] = run.v;
+    }
+    __syncthreads();
+    if (!colok) return;
+    V pre[VEC];
+#pragma unroll
+    for (int k = 0; k < VEC; ++k)
+        pre[k] = roff > 0 ? O::comb(s_carry[cg * VEC + k], sc[(roff - 1) * TCW + cg * VEC + k]) : s_carry[cg * VEC + k];
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+        const int64_t r = rbase + j;
+        if (r >= m) break;
+        if (VEC > 1) {
+            Vec16<T> o;
+#pragma unroll
+            for (int k = 0; k < VEC; ++k) {
+                const V z = O::comb(pre[k], a[j][k]);
+                o.e[k] = O::val(z);
+                if (OP == kArgmin) out_idx[r * w + c + k] = O::idx(z);
+            }
+            *reinterpret_cast<int4 *>(out + r * w + c) = *reinterpret_cast<const int4 *>(&o);
+        } else {
+            const V z = O::comb(pre[0], a[j][0]);
+            out[r * w + c] = O::val(z);
+            if (OP == kArgmin) out_idx[r * w + c] = O::idx(z);
+        }
+    }
+}
+
+// Few rows (m <= 8) of many columns, any alignment: a warp owns 4 x 32 consecutive columns, lane l
+// the columns l, l + 32, l + 64, l + 96 (every load and store instruction of the warp is one
+// contiguous 128-byte run), all m x 4 loads in flight, each column scanned down the rows.
+template <int OP, typename T, int MMAX>
+__global__ void __launch_bounds__(256)
+colscan_short_kernel(const T *__restrict__ x, int m, int64_t w, T *__restrict__ out, int64_t *__restrict__ out_idx) {
+    using O = Op<OP, T>;
+    using V = typename O::V;
+    constexpr int C = 4;
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (w + 32 * C - 1) / (32 * C);  // warp column groups
+    const int64_t wstride = (int64_t)gridDim.x * 8;
+    for (int64_t g = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5); g < nw; g += wstride) {
+        const int64_t c0 = g * 32 * C + lane;
+        T v[MMAX][C];
+#pragma unroll
+        for (int r = 0; r < MMAX; ++r)
+#pragma unroll
+            for (int k = 0; k < C; ++k)
+                if (r < m && c0 + 32 * k < w) v[r][k] = __ldg(x + (int64_t)r * w + c0 + 32 * k);
+#pragma unroll
+        for (int k = 0; k < C; ++k) {
+            const int64_t c = c0 + 32 * k;
+            if (c >= w) break;
+            V a = O::id();
+#pragma unroll
+            for (int r = 0; r < MMAX; ++r) {
+                if (r >= m) break;
+                a = O::comb(a, O::lift(v[r][k], r));
+                out[(int64_t)r * w + c] = O::val(a);
+                if (OP == kArgmin) out_idx[(int64_t)r * w + c] = O::idx(a);
+            }
+        }
+    }
+}
+
 struct ColScanPlan {
     int vec;
     bool narrow;  // colscan_narrow_kernel: a warp per row block
     int64_t WV, Y, rpu;
+    // one-pass look-back plan (taken whenever the rows must be split, Y > 1)
+    int CG, K;
+    int64_t ntx, nby, nblocks, nstate;
 };
+template <int OP, typename T> constexpr int colscan_lb_k() { return ScanShape<OP, T>::PACK ? 8 : 4; }
 static ColScanPlan colscan_plan(int dt, int64_t m, int64_t w, bool aligned) {
     ColScanPlan p;
     const int V = 16 / (int)dtype_size(dt);
@@ -2010,6 +2171,15 @@ static ColScanPlan colscan_plan(int dt, int64_t m, int64_t w, bool aligned) {
     p.Y = ceil_div(m, p.rpu);
     return p;
 }
+static void colscan_lb_plan(ColScanPlan &p, int64_t m, int K) {
+    p.K = K;
+    p.CG = (int)(p.WV < 32 ? p.WV : 32);
+    const int64_t RB = 256 / p.CG;
+    p.ntx = ceil_div(p.WV, p.CG);
+    p.nby = ceil_div(m, RB * K);
+    p.nblocks = p.ntx * p.nby;
+    p.nstate = p.nblocks * p.CG * p.vec;
+}
 
 template <int OP, typename T> struct ColScanRun {
     template <int VEC>
@@ -2017,6 +2187,24 @@ template <int OP, typename T> struct ColScanRun {
                         cudaStream_t st) {
         using V = typename Op<OP, T>::V;
         V *parts = (V *)((char *)ws + kWsHeader);
+        if (p.Y > 1) {  // rows split: the one-pass look-back kernel
+            ColScanPlan q = p;
+            colscan_lb_plan(q, m, colscan_lb_k<OP, T>());
+            using S = typename SOp<Op<OP, T>, false>::S;
+            using Sh = ScanShape<OP, T>;
+            char *b = (char *)ws + kWsHeader;
+            unsigned *counter = (unsigned *)b;
+            TileState<S, Sh::PACK> ts;
+            ts.w = (uint64_t *)(b + 256);
+            if constexpr (!Sh::PACK) {
+                ts.aggs = (S *)(b + 256 + scan_state_bytes(q.nstate));
+                ts.incls = ts.aggs + q.nstate;
+            }
+            if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(q.nstate), st) != cudaSuccess) return FS_ERR_CUDA;
+            colscan_lb_kernel<OP, T, VEC, colscan_lb_k<OP, T>()><<<(unsigned)q.nblocks, 256, 0, st>>>(
+                x, m, w, q.CG, q.ntx, counter, ts, out, out_idx);
+            return launch_status();
+        }
         if (p.narrow) {
             const unsigned gn = (unsigned)ceil_div(p.Y * 32, kColScanThreads);
             const int wv = (int)p.WV;
@@ -2058,6 +2246,17 @@ template <int OP, typename T> struct ColScanRun {
     }
     static fs_status run(const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx, void *ws, cudaStream_t st) {
         const bool aligned = ((uintptr_t)in & 15) == 0 && ((uintptr_t)out & 15) == 0;
+        const bool vec_ok = aligned && w % (16 / sizeof(T)) == 0;
+        if (m <= 8 && !vec_ok && w >= (int64_t)sm_count() * 2048) {  // few rows, many columns, any phase
+            const int64_t ng = ceil_div(w, 4 * 256);
+            const int64_t gmax = (int64_t)sm_count() * 16;
+            const unsigned grid = (unsigned)(ng < gmax ? ng : gmax);
+            if (m <= 4)
+                colscan_short_kernel<OP, T, 4><<<grid, 256, 0, st>>>((const T *)in, (int)m, w, (T *)out, out_idx);
+            else
+                colscan_short_kernel<OP, T, 8><<<grid, 256, 0, st>>>((const T *)in, (int)m, w, (T *)out, out_idx);
+            return launch_status();
+        }
         const ColScanPlan p = colscan_plan(sizeof(T) == 8 ? FS_I64 : FS_I32, m, w, aligned);
         if (p.vec > 1) return go<16 / sizeof(T)>(p, (const T *)in, m, w, (T *)out, out_idx, ws, st);
         return go<1>(p, (const T *)in, m, w, (T *)out, out_idx, ws, st);
@@ -2065,9 +2264,18 @@ template <int OP, typename T> struct ColScanRun {
 };
 
 size_t colscan_ws(int op, int dt, int64_t m, int64_t w) {
-    const ColScanPlan a = colscan_plan(dt, m, w, false), b = colscan_plan(dt, m, w, true);
+    ColScanPlan a = colscan_plan(dt, m, w, false), b = colscan_plan(dt, m, w, true);
     const int64_t Y = a.Y > b.Y ? a.Y : b.Y;
-    return kWsHeader + align_up((size_t)Y * w * acc_size(op, dt), 256);
+    // one-pass plan: counter, state words, and (not PACK) aggregate + inclusive payloads
+    const bool pack = op != FS_ARGMIN && dtype_size(dt) == 4;
+    const int K = pack ? 8 : 4;
+    colscan_lb_plan(a, m, K);
+    colscan_lb_plan(b, m, K);
+    const int64_t ns = a.nstate > b.nstate ? a.nstate : b.nstate;
+    const size_t pay = pack ? 0 : 2 * (size_t)ns * (acc_size(op, dt) + 8);
+    const size_t lb = 256 + scan_state_bytes(ns) + pay;
+    const size_t old = align_up((size_t)Y * w * acc_size(op, dt), 256);
+    return kWsHeader + (lb > old ? lb : old);
 }
 
 fs_status colscan_run(int op, int dt, const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx, void *ws,
