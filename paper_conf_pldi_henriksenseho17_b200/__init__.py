@@ -28,7 +28,8 @@ __all__ = [
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libfutseg.so")
+# FUTSEG_LIB: an alternative build of the same library (A/B measurement of build variants)
+_LIB_PATH = os.environ.get("FUTSEG_LIB") or os.path.join(_HERE, "libfutseg.so")
 
 if not os.path.exists(_LIB_PATH):
     raise ImportError(

@@ -1543,6 +1543,396 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
     return RG_KS_LOOKBACK;
 }
 
+// ---------------------------------------------------------------- ring scan (scanomap, long-row seg_scan)
+// The single pass of F5 (L1071-1074) with every tile kept ON CHIP between its read
+// and its write.  One CTA per SM streams tiles of 256 x kRingVPT 16-byte vectors
+// (36 KB) through a ring of kRingStages shared-memory slots; warps are specialised:
+//   producer warp  : next tile id from the atomic counter (increasing), 1-D TMA load
+//   aggregate group: (4 warps, tiles in order) the tile aggregate as soon as the tile
+//                    lands, published at once (status 1), so successors' look-backs
+//                    never wait on a tile that is merely queued in a ring
+//   consumer groups: (kRingNG x 8 warps, alternate tiles) scan the tile in registers
+//                    (thread-contiguous odd vector runs: conflict-free 16-byte shared
+//                    loads), warp 0 runs the decoupled look-back (32 x kRingEPL
+//                    predecessors per step) and publishes the inclusive prefix, then
+//                    prefix (+) local scan goes back into the slot and out with one TMA
+//                    bulk store.
+// Every element crosses HBM exactly once each way; nothing is re-read from L2.
+// Measured alternatives (tools/ring_trace.py, tools/scan_ab.py): separate look-back
+// warps started at the aggregate (0.75 of HBM: they start before their predecessors
+// are published and spin longer), wider look-back steps (worse), a third consumer
+// group or a store warp (no gain); the ring's bytes / slot hold time is the limit.
+// SEG: footnote 5's operator with the implicit flags i mod L == 0 (the look-back
+// stops at the first flagged predecessor).  ADD / MIN / MAX (ARGMIN keeps
+// scan_ws_kernel for its index output).
+#ifndef FS_RING_VPT
+#define FS_RING_VPT 9
+#endif
+#ifndef FS_RING_STAGES
+#define FS_RING_STAGES 6
+#endif
+#ifndef FS_RING_NG
+#define FS_RING_NG 2
+#endif
+#ifndef FS_RING_EPL
+#define FS_RING_EPL 1
+#endif
+constexpr int kRingEPL = FS_RING_EPL;  // look-back predecessors per lane per step
+#ifndef FS_RING_SLEEP
+#define FS_RING_SLEEP 0
+#endif
+constexpr int kRingSleep = FS_RING_SLEEP;  // ns between polls of an unpublished predecessor
+constexpr int kRingVPT = FS_RING_VPT, kRingStages = FS_RING_STAGES, kRingG = 256, kRingA = 128, kRingNG = FS_RING_NG;
+constexpr int kRingThreads = kRingNG * kRingG + kRingA + 32;
+static_assert(kRingVPT % 2 == 1, "odd vectors per thread: conflict-free 16-byte shared loads");
+template <int OP, typename T> struct RingShape {
+    static constexpr bool PACK = sizeof(T) == 4;
+    static constexpr int VEC = 16 / sizeof(T), E = kRingVPT * VEC;
+    static constexpr int64_t TILE = (int64_t)kRingG * E;
+    static constexpr unsigned TILE_BYTES = kRingG * kRingVPT * 16;
+    static constexpr unsigned SMEM = kRingStages * TILE_BYTES;
+};
+
+#ifdef FS_RING_TRACE
+// per-tile event times (%globaltimer, ns): issued, landed, aggregate published, prefix
+// published, written back, stored
+constexpr int kRingTraceTiles = 65536;
+__device__ unsigned long long g_ring_trace[kRingTraceTiles * 6];
+__device__ __forceinline__ void ring_mark(int64_t t, int e) {
+    unsigned long long v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+    if (t < kRingTraceTiles) g_ring_trace[t * 6 + e] = v;
+}
+extern "C" int fs_debug_ring_trace(void *host, size_t bytes) {
+    return (int)cudaMemcpyFromSymbol(host, g_ring_trace, bytes < sizeof(g_ring_trace) ? bytes : sizeof(g_ring_trace));
+}
+#define RING_MARK(t, e) ring_mark(t, e)
+#else
+#define RING_MARK(t, e)
+#endif
+
+template <int OP, typename T, bool SEG>
+__global__ void __launch_bounds__(kRingThreads, 1)
+scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__ out, const T *carry,
+                 unsigned *counter, TileState<typename SOp<Op<OP, T>, SEG>::S, RingShape<OP, T>::PACK> ts,
+                 int64_t ntiles) {
+    using O = Op<OP, T>;
+    using SO = SOp<O, SEG>;
+    using S = typename SO::S;
+    using Sh = RingShape<OP, T>;
+    constexpr int VEC = Sh::VEC, E = Sh::E, NST = kRingStages, NWG = kRingG / 32, NG = kRingNG;
+    constexpr int64_t TILE = Sh::TILE;
+    constexpr int T_AGG = NG * kRingG, T_PROD = T_AGG + kRingA;
+    constexpr int NMARK = NG;
+    static_assert(NMARK <= NST, "the end markers fit in the ring");
+    extern __shared__ __align__(128) unsigned char sbuf[];
+    // full: tile landed (TMA tx); aggd: aggregate published; empty: the aggregate group is
+    // done with the slot and the consumer's TMA store has read it
+    __shared__ uint64_t full[NST], aggd[NST], empty[NST];
+    __shared__ int64_t s_tid[NST];
+    __shared__ S s_wtot[NG][NWG], s_wpre[NG][NWG];
+    __shared__ typename O::V s_ared[2][kRingA / 32];
+    const int tid = threadIdx.x, lane = tid & 31;
+    if (tid == 0) {
+        for (int s = 0; s < NST; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&aggd[s], 1);
+            mbar_init(&empty[s], 2);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    auto tile_len = [&](int64_t t, int64_t &nv, int64_t &nbulk) {
+        nv = (n - t * TILE) < TILE ? (n - t * TILE) : TILE;
+        nbulk = ((nv * (int64_t)sizeof(T)) & ~(int64_t)15) / (int64_t)sizeof(T);
+    };
+    if (tid >= T_PROD) {  // ---- producer warp: tile ids in increasing order, TMA into the ring
+        if (lane == 0) {
+            int marks = 0;
+            for (int64_t k = 0; marks < NMARK; ++k) {
+                const int s = (int)(k % NST);
+                if (k >= NST) mbar_wait(&empty[s], (unsigned)((k / NST) - 1) & 1u);
+                const int64_t t = marks ? ntiles : (int64_t)atomicAdd(counter, 1u);
+                if (t >= ntiles) {  // NMARK end markers in consecutive slots: every round-robin
+                    s_tid[s] = -1;  // member of every role meets one
+                    ++marks;
+                    mbar_arrive(&full[s]);
+                    continue;
+                }
+                s_tid[s] = t;
+                RING_MARK(t, 0);
+                int64_t nv, nbulk;
+                tile_len(t, nv, nbulk);
+                if (nbulk) {
+                    mbar_expect_tx(&full[s], (unsigned)(nbulk * (int64_t)sizeof(T)));
+                    tma_load_1d(sbuf + (size_t)s * Sh::TILE_BYTES, in + t * TILE,
+                                (unsigned)(nbulk * (int64_t)sizeof(T)), &full[s]);
+                } else {
+                    mbar_arrive(&full[s]);
+                }
+            }
+        }
+        return;
+    }
+    if (tid >= T_AGG) {  // ---- aggregate group: every tile's aggregate as soon as it lands, in order
+        const int at = tid - T_AGG, aw = at >> 5;
+        for (int64_t k = 0, marks = 0; marks < NMARK; ++k) {
+            const int s = (int)(k % NST);
+            mbar_wait(&full[s], (unsigned)(k / NST) & 1u);
+            const int64_t t = s_tid[s];
+            if (t < 0) {
+                ++marks;
+                continue;
+            }
+            if (at == 0) RING_MARK(t, 1);
+            const int64_t t0 = t * TILE;
+            int64_t nv, nbulk;
+            tile_len(t, nv, nbulk);
+            const unsigned char *slot = sbuf + (size_t)s * Sh::TILE_BYTES;
+            // SEG: the elements after the tile's last segment start (closed form), flag = a start exists
+            int64_t lo = 0;
+            int f = 0;
+            if constexpr (SEG) {
+                const int64_t r = t0 % L, i0 = r == 0 ? 0 : L - r;
+                if (i0 < nv) {
+                    lo = i0 + ((nv - 1 - i0) / L) * L;
+                    f = 1;
+                }
+            }
+            typename O::V acc = O::id();
+            if (nv == TILE && lo == 0) {
+#pragma unroll
+                for (int j = 0; j < 2 * kRingVPT; ++j) {
+                    const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((j * kRingA + at) << 4)));
+#pragma unroll
+                    for (int q = 0; q < VEC; ++q) acc = O::comb(acc, a.e[q]);
+                }
+            } else {
+                for (int j = 0; j < 2 * kRingVPT; ++j) {
+                    const int64_t e = (int64_t)(j * kRingA + at) * VEC;
+#pragma unroll
+                    for (int q = 0; q < VEC; ++q) {
+                        const int64_t p = e + q;
+                        if (p >= lo && p < nv)
+                            acc = O::comb(acc, p < nbulk ? reinterpret_cast<const T *>(slot)[p] : in[t0 + p]);
+                    }
+                }
+            }
+#pragma unroll
+            for (int m = 16; m > 0; m >>= 1) acc = O::comb(acc, shfl_xor(acc, m));
+            if ((at & 31) == 0) s_ared[k & 1][aw] = acc;
+            named_bar(1 + NG, kRingA);
+            if (at == 0) {
+                S agg{s_ared[k & 1][0], f};
+#pragma unroll
+                for (int w = 1; w < kRingA / 32; ++w) agg.v = O::comb(agg.v, s_ared[k & 1][w]);
+                if (t > 0) ts.publish(t, agg, kStAgg);
+                RING_MARK(t, 2);
+                mbar_arrive(&aggd[s]);
+                mbar_arrive(&empty[s]);
+            }
+        }
+        return;
+    }
+    // ---- consumer group g: tiles k = g, g + NG, ...
+    const int g = tid / kRingG, gt = tid % kRingG, warp = gt >> 5;
+    for (int64_t k = g;; k += NG) {
+        const int s = (int)(k % NST);
+        mbar_wait(&full[s], (unsigned)(k / NST) & 1u);
+        const int64_t t = s_tid[s];
+        if (t < 0) break;
+        const int64_t t0 = t * TILE;
+        int64_t nv, nbulk;
+        tile_len(t, nv, nbulk);
+        unsigned char *slot = sbuf + (size_t)s * Sh::TILE_BYTES;
+        const int e0 = gt * E;  // this thread's first element in the tile
+        // local inclusive scan of the thread's E contiguous elements, in registers
+        T x[E];
+        if (nv == TILE) {
+#pragma unroll
+            for (int j = 0; j < kRingVPT; ++j) {
+                const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((gt * kRingVPT + j) << 4)));
+#pragma unroll
+                for (int q = 0; q < VEC; ++q) x[j * VEC + q] = a.e[q];
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                const int64_t p = e0 + i;
+                x[i] = p < nbulk ? reinterpret_cast<const T *>(slot)[p] : (p < nv ? in[t0 + p] : O::id());
+            }
+        }
+        int64_t r0 = 0;
+        if constexpr (SEG) r0 = (t0 + e0) % L;
+        // no segment start among this thread's elements: the plain scan (flag 0)
+        const bool noflag = !SEG || (r0 != 0 && L - r0 >= E);
+        S run = SO::id();
+        if (noflag) {
+#pragma unroll
+            for (int i = 0; i < E; ++i) run.v = O::comb(run.v, x[i]);
+        } else {
+            int64_t r = r0;
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                S e;
+                e.v = x[i];
+                e.f = SEG ? (r == 0) : 0;
+                if (SEG) {
+                    ++r;
+                    if (r == L) r = 0;
+                }
+                run = SO::comb(run, e);
+            }
+        }
+        // ordered inclusive warp scan of the thread totals
+        S a = run;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const S o = SO::up(a, off);
+            if (lane >= off) a = SO::comb(o, a);
+        }
+        S tex = SO::up(a, 1);
+        if (lane == 0) tex = SO::id();
+        if (lane == 31) s_wtot[g][warp] = a;
+        named_bar(1 + g, kRingG);
+        if (warp == 0) {
+            S w = lane < NWG ? s_wtot[g][lane] : SO::id();
+#pragma unroll
+            for (int off = 1; off < NWG; off <<= 1) {
+                const S o = SO::up(w, off);
+                if (lane >= off) w = SO::comb(o, w);
+            }
+            S wex = SO::up(w, 1);
+            if (lane == 0) wex = SO::id();
+            const S agg = SO::bcast(w, NWG - 1);
+            // decoupled look-back over the published predecessors
+            S exc = SO::id();
+            if (t == 0) {
+                if (carry) exc = S{O::lift(*carry, -1), 0};
+            } else {
+                    // wide look-back: lane i polls predecessors j - EPL*i - 0 .. EPL-1 (all loads of a
+                    // step in flight together: 32*EPL predecessors per L2 round trip)
+                    constexpr int EPL = kRingEPL;
+                    int64_t j = t - 1;
+                    while (true) {
+                        S v[EPL];
+                        unsigned st[EPL];
+    #pragma unroll
+                        for (int e = 0; e < EPL; ++e) {
+                            const int64_t idx = j - (int64_t)EPL * lane - e;
+                            v[e] = SO::id();
+                            st[e] = idx >= 0 ? ts.poll(idx, v[e]) : kStIncl;
+                        }
+    #pragma unroll
+                        for (int e = 0; e < EPL; ++e) {
+                            const int64_t idx = j - (int64_t)EPL * lane - e;
+                            while (st[e] == 0) {
+                                if (kRingSleep) __nanosleep(kRingSleep);
+                                st[e] = ts.poll(idx, v[e]);
+                            }
+                        }
+                        // this lane's nearest inclusive prefix (idx < 0 counts as one: nothing left)
+                        int ne = EPL;
+    #pragma unroll
+                        for (int e = EPL - 1; e >= 0; --e)
+                            if (st[e] == kStIncl) ne = e;
+                        const unsigned m = __ballot_sync(0xffffffffu, ne < EPL);
+                        const int kk = m ? __ffs(m) - 1 : 32;
+                        // the lane's ordered fold of its entries up to (and including) its nearest
+                        // inclusive prefix; entries further left are farther back
+                        S a = SO::id();
+    #pragma unroll
+                        for (int e = EPL - 1; e >= 0; --e) {
+                            const int64_t idx = j - (int64_t)EPL * lane - e;
+                            if (e <= ne && idx >= 0) a = SO::comb(a, v[e]);
+                        }
+                        if (lane > kk) a = SO::id();
+                        // ordered reduction: higher lanes are further left
+    #pragma unroll
+                        for (int off = 1; off < 32; off <<= 1) {
+                            const S o = SO::down(a, off);
+                            if (lane + off < 32) a = SO::comb(o, a);
+                        }
+                        exc = SO::comb(SO::bcast(a, 0), exc);
+                        if (m || j < 32 * EPL || (SEG && exc.f)) break;
+                        j -= 32 * EPL;
+                    }
+            }
+            // (after the aggregate group's publish: never downgrade an inclusive prefix)
+            mbar_wait(&aggd[s], (unsigned)(k / NST) & 1u);
+            if (lane == 0) {
+                ts.publish(t, SO::comb(exc, agg), kStIncl);
+                RING_MARK(t, 3);
+            }
+            if (lane < NWG) s_wpre[g][lane] = SO::comb(exc, wex);
+        }
+        named_bar(1 + g, kRingG);
+        const S p = SO::comb(s_wpre[g][warp], tex);
+        if (noflag) {
+            typename O::V c = p.v;
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                c = O::comb(c, x[i]);
+                x[i] = O::val(c);
+            }
+        } else {
+            S c = p;
+            int64_t r = r0;
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                S e;
+                e.v = x[i];
+                e.f = SEG ? (r == 0) : 0;
+                if (SEG) {
+                    ++r;
+                    if (r == L) r = 0;
+                }
+                c = SO::comb(c, e);
+                x[i] = O::val(c.v);
+            }
+        }
+        if (nv == TILE) {
+#pragma unroll
+            for (int j = 0; j < kRingVPT; ++j) {
+                Vec16<T> v;
+#pragma unroll
+                for (int q = 0; q < VEC; ++q) v.e[q] = x[j * VEC + q];
+                int4 w;
+                memcpy(&w, &v, 16);
+                *reinterpret_cast<int4 *>(slot + ((gt * kRingVPT + j) << 4)) = w;
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < E; ++i) {
+                const int64_t q = e0 + i;
+                if (q < nbulk) reinterpret_cast<T *>(slot)[q] = x[i];
+                else if (q < nv) out[t0 + q] = x[i];
+            }
+        }
+        fence_proxy_async();
+        named_bar(1 + g, kRingG);
+        if (gt == 0) {
+            RING_MARK(t, 4);
+            if (nbulk) {
+                tma_store_1d(out + t0, slot, (unsigned)(nbulk * (int64_t)sizeof(T)));
+                bulk_commit();
+                bulk_wait_read<0>();
+            }
+            RING_MARK(t, 5);
+            mbar_arrive(&empty[s]);
+        }
+    }
+    if (gt == 0) bulk_wait<0>();
+}
+
+// FUTSEG_SCAN_KERNEL=ws selects the slab scan instead of the ring scan (A/B measurement only)
+static bool scan_ring_disabled() {
+    static const int v = [] {
+        const char *e = getenv("FUTSEG_SCAN_KERNEL");
+        return (e && e[0] == 'w' && e[1] == 's') ? 1 : 0;
+    }();
+    return v != 0;
+}
 template <int OP, typename T> struct ScanRun {
     template <bool NN, bool SEG, bool TMA>
     static fs_status go(const void *in0, const void *in1, int64_t n, int64_t L, const fs_mapdesc &map, void *out,
@@ -1558,6 +1948,30 @@ template <int OP, typename T> struct ScanRun {
         if constexpr (!Sh::PACK) {
             ts.aggs = (S *)(b + 256 + scan_state_bytes(ntiles));
             ts.incls = ts.aggs + ntiles;
+        }
+        if constexpr (TMA && !NN && OP != kArgmin) {  // the ring scan (16-byte aligned buffers)
+            if (!scan_ring_disabled()) {
+                using ShR = RingShape<OP, T>;
+                const int64_t ntr = ceil_div(n, ShR::TILE);
+                if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntr), st) != cudaSuccess) return FS_ERR_CUDA;
+                TileState<S, ShR::PACK> tr;
+                tr.w = ts.w;
+                if constexpr (!ShR::PACK) {
+                    tr.aggs = ts.aggs;
+                    tr.incls = ts.incls;
+                }
+                auto kr = scan_ring_kernel<OP, T, SEG>;
+                static bool attr = false;
+                if (!attr) {
+                    cudaFuncSetAttribute((const void *)kr, cudaFuncAttributeMaxDynamicSharedMemorySize, ShR::SMEM);
+                    attr = true;
+                }
+                const int64_t G0 = sm_count();
+                const int64_t G = ntr < G0 ? ntr : G0;
+                kr<<<(unsigned)(G > 0 ? G : 1), kRingThreads, ShR::SMEM, st>>>((const T *)in0, n, L, (T *)out,
+                                                                               (const T *)carry, counter, tr, ntr);
+                return launch_status();
+            }
         }
         if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntiles), st) != cudaSuccess) return FS_ERR_CUDA;
         if constexpr (TMA && !NN) {  // the warp-specialised slab scan (16-byte aligned buffers)

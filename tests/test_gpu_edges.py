@@ -344,3 +344,57 @@ def test_full_c5_transpose_blocks_vs_oracle(fs):
     # a ragged block too (odd offset and width)
     want = oracle.transpose_2d(host(x[777:777 + 33, 5:5 + 1001]))
     np.testing.assert_array_equal(host(t[5:5 + 1001, 777:777 + 33]), want)
+
+
+# ------------------------------------------------------------------ ring scan tile edges
+# scan_ring_kernel (scanomap and the segmented look-back scan on 16-byte aligned buffers,
+# add/min/max): tiles of 256 x 9 16-byte vectors = 9216 four-byte / 4608 eight-byte elements.
+RING_TILE = {4: 9216, 8: 4608}
+
+
+@pytest.mark.parametrize("dt", [np.int32, np.int64, np.float32])
+@pytest.mark.parametrize("op", ["add", "min", "max"])
+def test_scanomap_ring_tile_edges(fs, dt, op):
+    """Sizes one element around a tile, a ragged sub-vector tail, one tile short of and just
+    past a whole ring of tiles per SM, and a carry-in continuing a previous scan (F5)."""
+    t = RING_TILE[np.dtype(dt).itemsize]
+    for n in (1, 3, t - 1, t, t + 1, t + 3, 2 * t + 2, 6 * 148 * t - 1, 6 * 148 * t + 5):
+        if np.dtype(dt).kind == "i":
+            x = wrap_input(n, n % 89, dt, op)
+        else:
+            x = workloads.mixed(n, n % 89, dt)
+        got = fs.scanomap(cu(x), op)
+        want = oracle.scan(x, op)
+        if dt == np.float32 and op == "add":
+            asum = oracle.scan(np.abs(x), "add")
+            assert np.all(np.abs(host(got).astype(np.float64) - want) <= 1e-4 * asum + 1e-30), n
+        else:
+            eq(got, want, f"ring scan {np.dtype(dt).name} {op} n={n}")
+    if op == "add" and np.dtype(dt).kind == "i":
+        x = workloads.full_range(5 * t + 7, 11, dt)
+        h = 2 * t + 1
+        a = fs.scanomap(cu(x[:h]), "add")
+        b = fs.scanomap(cu(x[h:]), "add", carry=a[-1:].clone())
+        eq(torch.cat([a, b]), oracle.scan(x, "add"), "ring scan carry")
+
+
+@pytest.mark.parametrize("dt", [np.int32, np.int64, np.float32])
+def test_seg_scan_ring_rows_around_tile(fs, dt):
+    """Segmented ring scan: rows shorter than, equal to and longer than a tile, row starts
+    inside and at tile boundaries (the look-back stops at the first flagged predecessor)."""
+    t = RING_TILE[np.dtype(dt).itemsize]
+    fs.force_seg_regime(5)
+    try:
+        for nseg, L in ((40, t - 1), (30, t), (20, t + 1), (7, 3 * t + 5), (3, 40 * t + 1)):
+            for op in ("add", "max"):
+                x = workloads.full_range(nseg * L, L, dt) if np.dtype(dt).kind == "i" else \
+                    workloads.mixed(nseg * L, L, dt)
+                got = fs.seg_scan(cu(x), nseg, L, op)
+                want = oracle.seg_scan(x, nseg, L, op)
+                if dt == np.float32 and op == "add":
+                    asum = oracle.seg_scan(np.abs(x), nseg, L, "add")
+                    assert np.all(np.abs(host(got).astype(np.float64) - want) <= 1e-4 * asum + 1e-30)
+                else:
+                    eq(got, want, f"ring seg_scan {np.dtype(dt).name} {op} {nseg}x{L}")
+    finally:
+        fs.force_seg_regime(-1)
