@@ -320,8 +320,11 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *   2 = KG3 block per segment                                           fs_seg_reduce
  *   3 = KG4 several blocks per segment, partials combined by the last   fs_seg_reduce
  *   4 = column kernels (FS_COL_MAJOR with nseg > 1 and seglen > 1)      both
- *   5 = single-pass segmented decoupled-look-back slab scan (the general
- *       case: argmin, carries, misaligned buffers, lengths no other regime takes)
+ *   5 = single-pass segmented decoupled-look-back scan (the general case: argmin,
+ *       carries, misaligned buffers, lengths no other regime takes; long rows with fewer
+ *       than 1.7 x SMs rows).  add/min/max on 16-byte aligned buffers run the ring scan
+ *       (tiles held in a shared-memory TMA ring between read and write), argmin the slab
+ *       scan
  *   6 = empty input (nseg == 0 or seglen == 0: neutral fill / nothing)  both
  *   7 = KS0 power-of-two rows of <= 256 16-byte vectors (seglen <= 1024 f32/i32,
  *       512 i64), 16-byte aligned buffers: in-register + shuffle scan, a shared-memory
@@ -331,9 +334,9 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       when forced (fs_force_seg_regime): KS3's TMA ring is the plan's choice for these
  *       rows since round 2 (L = 3: 0.57 -> 0.83 of the HBM roofline)
  *   9 = KS2 rows of >= 4 chunks of 256 x R vectors (12288 f32/i32 add/min/max, 4096
- *       argmin, 2048 i64) when there are at least as many rows as SMs (in/out with the
- *       same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with a
- *       running carry (no look-back)
+ *       argmin, 2048 i64) when there are at least 1.7 x as many rows as SMs (in/out with
+ *       the same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with
+ *       a running carry (no look-back)
  *  10 = KS0-BIG power-of-two rows of 2-8 CTA steps (256 < seglen/VEC <= 2048: 2048..8192
  *       f32/i32, 1024..4096 i64), 16-byte aligned: a CTA loads a whole row per step,
  *       warp 0 scans the warp totals
@@ -343,8 +346,8 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       a 3-slot ring and TMA bulk stores when both buffers are 16-byte aligned and a tile
  *       of R rows is <= 72 KB), odd-length per-thread pieces, a CTA scan of the piece
  *       summaries (no look-back)
- *  12 = flat (unsegmented) slab scan per row: one row (nseg == 1), or fewer rows than SMs
- *       of >= 2^26 elements each, 16-byte aligned
+ *  12 = flat (unsegmented) scan per row: one row (nseg == 1); several rows only when
+ *       forced (16-byte aligned; regime 5 is faster for a few long rows)
  * fs_seg_regime returns the regime a call with these sizes takes on the current device
  * when its buffers come from an allocator (16-byte aligned); misaligned views may take
  * 5 instead.  The row-major seg_scan plan is one function shared with the dispatcher.
@@ -359,7 +362,7 @@ int32_t fs_last_seg_regime(void);
 /* Testing / sweep aid: force a regime for subsequent calls in this process; -1
  * restores automatic selection.  0..3 force the FS_ROW_MAJOR seg_reduce regime;
  * 5 and 7..12 force a row-major seg_scan regime wherever its preconditions above hold
- * (elsewhere the automatic choice stands; forced 12 drops its 2^26 length threshold).
+ * (elsewhere the automatic choice stands).
  * Also settable with the environment variable FUTSEG_FORCE_REGIME.  Returns
  * FS_ERR_UNSUPPORTED for other values. */
 fs_status fs_force_seg_regime(int32_t regime);

@@ -1497,13 +1497,17 @@ segscan_cta_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *__restri
 // (seg sweep, profiles/r01_seg_sweep.json: at >= 1 row per SM KS2 beats the segmented look-back scan,
 // 256-268 rows 3.8 -> 4.8 TB/s, 512 rows 3.8 -> 4.5; below one row per SM SMs idle: 128 rows 3.6, 32 rows 1.1)
 #ifndef FS_KS2_MINF
-#define FS_KS2_MINF 85  // rows >= 0.85 x SMs: 128 rows of 2^21 0.736 (look-back) -> 0.751; 64 rows 0.41
+// rows >= 1.7 x SMs (profiles/r02_scan_regimes.jsonl): KS2 0.94-0.98 of HBM from 256 rows up; at
+// 128 rows of 2^21 KS2 0.78 vs the ring look-back scan 0.87
+#define FS_KS2_MINF 170
 #endif
 static bool nseg_ok(int64_t n, int64_t L) { return L > 0 && n / L >= (int64_t)sm_count() * FS_KS2_MINF / 100; }
 #ifndef FS_FLAT_ROW_MIN
-#define FS_FLAT_ROW_MIN (1 << 26)
+#define FS_FLAT_ROW_MIN INT64_MAX
 #endif
-constexpr int64_t kFlatRowMin = FS_FLAT_ROW_MIN;  // rows at least this long and fewer than the SMs: flat scan per row
+// rows at least this long: flat scan per row.  Off by default since the ring look-back scan
+// (0.87 at 2 and 4 rows, one launch) beats one ring launch per row (0.86 / 0.78); forceable (12).
+constexpr int64_t kFlatRowMin = FS_FLAT_ROW_MIN;
 template <int OP, typename T> constexpr int ks2_rows() { return (sizeof(T) == 4 && OP != kArgmin) ? 3 : 1; }
 template <typename T> constexpr int dt_of() {
     return sizeof(T) == 8 ? FS_I64 : (std::is_same<T, float>::value ? FS_F32 : FS_I32);

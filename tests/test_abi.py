@@ -215,7 +215,7 @@ def test_workspace_queries_and_regimes(fs):
     assert r(1 << 12, 2048, scan=True) == 10 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 10
     assert r(1 << 12, 8192, scan=True) == 10 and r(1 << 12, 16384, scan=True, dtype=torch.int64) == 9
     assert r(1 << 20, 512, scan=True, dtype=torch.int64) == 7 and r(1 << 20, 1024, scan=True, dtype=torch.int64) == 10
-    assert r(1, 1 << 28, scan=True) == 12 and r(2, 1 << 27, scan=True) == 12 and r(1, 5, scan=True) == 12
+    assert r(1, 1 << 28, scan=True) == 12 and r(2, 1 << 27, scan=True) == 5 and r(1, 5, scan=True) == 12
     assert r(4096, 1000, scan=True, op="argmin") == 5 and r(1 << 21, 128, scan=True, op="argmin") == 7
     assert r(0, 64) == 6 and r(64, 0) == 6
     assert r(64, 64, dtype=torch.int64, op="argmin") == 0
