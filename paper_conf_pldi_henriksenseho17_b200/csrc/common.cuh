@@ -251,6 +251,12 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
     }
 }
 
+// L2 prefetch of a contiguous global range (no shared memory, no completion): issued a few
+// stages ahead of the TMA load that will read it, it moves the HBM latency off the ring slot
+__device__ __forceinline__ void prefetch_l2_bulk(const void *src, unsigned bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
 // 1-D bulk copy shared -> global (SASS UBLKCP), tracked by bulk async-groups of the
 // issuing thread: commit after issuing, wait_group_read<N> before the source smem
 // is overwritten (all but the N most recent groups have finished READING smem),

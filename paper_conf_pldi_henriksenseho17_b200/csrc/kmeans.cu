@@ -60,6 +60,7 @@ constexpr int kKmK = 32;       // max clusters
 constexpr int kKmMaxD = 40;
 constexpr int kKmSeg = 16;     // stages per D2 buffer
 
+
 __device__ __forceinline__ uint32_t km_smem(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void km_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(km_smem(bar)) : "memory");
@@ -768,16 +769,23 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
     int *pcnt = (int *)(w + kWsHeader + align_up((size_t)G * k * d * 4, 256));
     int NR, NX;
     km_rings(d, NC, NR, NX);
-    {
+    {   // debug switches (tools/km_trace.py, tools/km_skip.py): set once per process and device,
+        // only when requested (the device globals default to off: no copies on the product path)
+        static const char *e = getenv("FUTSEG_KM_TRACE");
+        static const int skip = getenv("FUTSEG_KM_SKIP") ? atoi(getenv("FUTSEG_KM_SKIP")) : 0;
         static long long *tr = nullptr;
-        const char *e = getenv("FUTSEG_KM_TRACE");
-        if (e && !tr) cudaMalloc(&tr, 16 * 8 * 8192);
-        long long *p = e ? tr : nullptr;
-        cudaMemcpyToSymbolAsync(g_km_trace, &p, sizeof(p), 0, cudaMemcpyHostToDevice, st);
-        static int cta = e ? atoi(e) : 0;
-        cudaMemcpyToSymbolAsync(g_km_trace_cta, &cta, sizeof(cta), 0, cudaMemcpyHostToDevice, st);
-        static int skip = getenv("FUTSEG_KM_SKIP") ? atoi(getenv("FUTSEG_KM_SKIP")) : 0;
-        cudaMemcpyToSymbolAsync(g_km_skip, &skip, sizeof(skip), 0, cudaMemcpyHostToDevice, st);
+        static unsigned done_dev = 0;
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if ((e || skip) && dev < 32 && !(done_dev & (1u << dev))) {
+            if (e && !tr) cudaMalloc(&tr, 16 * 8 * 8192);
+            long long *p = e ? tr : nullptr;
+            const int cta = e ? atoi(e) : 0;
+            cudaMemcpyToSymbol(g_km_trace, &p, sizeof(p));
+            cudaMemcpyToSymbol(g_km_trace_cta, &cta, sizeof(cta));
+            cudaMemcpyToSymbol(g_km_skip, &skip, sizeof(skip));
+            done_dev |= 1u << dev;
+        }
     }
     const size_t smem = km_smem_bytes(d, NC, NR, NX);
     auto kern = kmeans_tc_kernel<NC, DT>;

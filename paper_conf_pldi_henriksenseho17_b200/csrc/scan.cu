@@ -1551,7 +1551,11 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
 // The single pass of F5 (L1071-1074) with every tile kept ON CHIP between its read
 // and its write.  One CTA per SM streams tiles of 256 x kRingVPT 16-byte vectors
 // (36 KB) through a ring of kRingStages shared-memory slots; warps are specialised:
-//   producer warp  : next tile id from the atomic counter (increasing), 1-D TMA load
+//   producer warp  : tile ids from the atomic counter (increasing), taken kRingPf = 1 tile
+//                    ahead and prefetched into L2 (cp.async.bulk.prefetch.L2) so that the
+//                    1-D TMA load into a freed slot hits L2: the slot no longer waits on HBM
+//                    latency (scanomap 0.89 -> 0.99 of the HBM peak; 2 or 4 ahead hold ids
+//                    longer before their aggregates can be published: 0.97 / 0.91)
 //   aggregate group: (4 warps, tiles in order) the tile aggregate as soon as the tile
 //                    lands, published at once (status 1), so successors' look-backs
 //                    never wait on a tile that is merely queued in a ring
@@ -1562,7 +1566,7 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
 //                    prefix (+) local scan goes back into the slot and out with one TMA
 //                    bulk store.
 // Every element crosses HBM exactly once each way; nothing is re-read from L2.
-// Measured alternatives (tools/ring_trace.py, tools/scan_ab.py): separate look-back
+// Other measured alternatives (tools/ring_trace.py, tools/scan_ab.py): separate look-back
 // warps started at the aggregate (0.75 of HBM: they start before their predecessors
 // are published and spin longer), wider look-back steps (worse), a third consumer
 // group or a store warp (no gain); the ring's bytes / slot hold time is the limit.
@@ -1582,6 +1586,10 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
 #define FS_RING_EPL 1
 #endif
 constexpr int kRingEPL = FS_RING_EPL;  // look-back predecessors per lane per step
+#ifndef FS_RING_PF
+#define FS_RING_PF 1
+#endif
+constexpr int kRingPf = FS_RING_PF;  // tile ids taken (and L2-prefetched) ahead of the ring
 #ifndef FS_RING_SLEEP
 #define FS_RING_SLEEP 0
 #endif
@@ -1653,10 +1661,42 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
     if (tid >= T_PROD) {  // ---- producer warp: tile ids in increasing order, TMA into the ring
         if (lane == 0) {
             int marks = 0;
+            // kRingPf tile ids taken ahead and prefetched into L2 (the ring slot then waits on an
+            // L2 hit instead of HBM latency)
+            int64_t q[kRingPf > 0 ? kRingPf : 1];
+            int qh = 0, qn = 0;
+            bool dry = false;
+            auto take = [&]() {
+                if (dry) return;
+                const int64_t u = (int64_t)atomicAdd(counter, 1u);
+                if (u >= ntiles) {
+                    dry = true;
+                    return;
+                }
+                q[(qh + qn) % kRingPf] = u;
+                ++qn;
+                int64_t nv, nbulk;
+                tile_len(u, nv, nbulk);
+                if (nbulk) prefetch_l2_bulk(in + u * TILE, (unsigned)(nbulk * (int64_t)sizeof(T)));
+            };
+            if (kRingPf > 0)
+                for (int i = 0; i < kRingPf; ++i) take();
             for (int64_t k = 0; marks < NMARK; ++k) {
                 const int s = (int)(k % NST);
                 if (k >= NST) mbar_wait(&empty[s], (unsigned)((k / NST) - 1) & 1u);
-                const int64_t t = marks ? ntiles : (int64_t)atomicAdd(counter, 1u);
+                int64_t t;
+                if (kRingPf > 0) {
+                    if (qn > 0) {
+                        t = q[qh];
+                        qh = (qh + 1) % kRingPf;
+                        --qn;
+                        take();
+                    } else {
+                        t = ntiles;
+                    }
+                } else {
+                    t = marks ? ntiles : (int64_t)atomicAdd(counter, 1u);
+                }
                 if (t >= ntiles) {  // NMARK end markers in consecutive slots: every round-robin
                     s_tid[s] = -1;  // member of every role meets one
                     ++marks;

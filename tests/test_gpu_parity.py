@@ -619,10 +619,10 @@ def test_seg_scan_rows_ks3(fs, nseg, seglen, offset):
         assert_reduced(got, want, op, asum, f"segscan ks3 {nseg}x{seglen}+{offset} {dt.__name__} {op}")
 
 
-@pytest.mark.parametrize("nseg,seglen", [(149, 3 * 8192 + 4), (300, 20_000), (150, 65_536), (1000, 12_292)])
+@pytest.mark.parametrize("nseg,seglen", [(253, 3 * 8192 + 4), (300, 20_000), (256, 65_536), (1000, 12_292)])
 def test_seg_scan_row_stream(fs, nseg, seglen):
-    """KS2 through the TMA ring (regime 9, 16-byte aligned, seglen a multiple of the vector):
-    rows of several 8192-element tiles and a partial last tile, equal rows per CTA; add/min/max
+    """KS2 through the TMA ring (regime 9: >= 1.7 x SMs rows, 16-byte aligned, seglen a multiple
+    of the vector): rows of several 8192-element tiles and a partial last tile; add/min/max
     on every dtype, int wrap-around."""
     for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int64, "min"), (np.int64, "add"),
                    (np.int32, "max"), (np.float32, "min")):
