@@ -321,10 +321,11 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *   3 = KG4 several blocks per segment, partials combined by the last   fs_seg_reduce
  *   4 = column kernels (FS_COL_MAJOR with nseg > 1 and seglen > 1)      both
  *   5 = single-pass segmented decoupled-look-back scan (the general case: argmin,
- *       carries, misaligned buffers, lengths no other regime takes; long rows with fewer
- *       than 1.7 x SMs rows).  add/min/max on 16-byte aligned buffers run the ring scan
- *       (tiles held in a shared-memory TMA ring between read and write), argmin the slab
- *       scan
+ *       carries, misaligned buffers, lengths no other regime takes).  add/min/max on
+ *       16-byte aligned buffers run the ring scan (tiles held in a shared-memory TMA ring
+ *       between read and write) and take every row longer than 4096 elements that KS2
+ *       cannot stream by TMA (fewer than 1.7 x SMs rows, or L not a multiple of the
+ *       16-byte vector); argmin runs the slab scan
  *   6 = empty input (nseg == 0 or seglen == 0: neutral fill / nothing)  both
  *   7 = KS0 power-of-two rows of <= 256 16-byte vectors (seglen <= 1024 f32/i32,
  *       512 i64), 16-byte aligned buffers: in-register + shuffle scan, a shared-memory
@@ -335,12 +336,14 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       rows since round 2 (L = 3: 0.57 -> 0.83 of the HBM roofline)
  *   9 = KS2 rows of >= 4 chunks of 256 x R vectors (12288 f32/i32 add/min/max, 4096
  *       argmin, 2048 i64) when there are at least 1.7 x as many rows as SMs (in/out with
- *       the same 16-byte phase): a CTA owns whole rows and scans them chunk by chunk with
- *       a running carry (no look-back)
+ *       the same 16-byte phase; add/min/max on aligned buffers only when L is a multiple
+ *       of the vector, streamed by TMA): a CTA owns whole rows and scans them chunk by
+ *       chunk with a running carry (no look-back)
  *  10 = KS0-BIG power-of-two rows of 2-8 CTA steps (256 < seglen/VEC <= 2048: 2048..8192
  *       f32/i32, 1024..4096 i64), 16-byte aligned: a CTA loads a whole row per step,
  *       warp 0 scans the warp totals
- *  11 = KS3 rows of 32 < seglen <= 16384 (8192 for i64), op != ARGMIN, element-aligned,
+ *  11 = KS3 rows of 32 < seglen <= 16384 (8192 for i64; 4096 when the ring scan can run),
+ *       op != ARGMIN, element-aligned,
  *       and rows of 2..32 elements (not powers of two) with 16-byte aligned input and
  *       output: R whole rows per CTA staged in shared memory (by TMA bulk copies through
  *       a 3-slot ring and TMA bulk stores when both buffers are 16-byte aligned and a tile

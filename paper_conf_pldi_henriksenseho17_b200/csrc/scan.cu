@@ -1524,6 +1524,11 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
     const int64_t es = (int64_t)dtype_size(dt), VEC = 16 / es;
     const bool pow2 = (L & (L - 1)) == 0;
     const int64_t ks2ch = 256 * VEC * ((es == 4 && op != FS_ARGMIN) ? 3 : 1);
+    // (preconditions; a forced regime needs only these.  Preference:) the ring scan (regime 5
+    // on 16-byte aligned buffers, add/min/max) beats KS3 above 4096
+    // elements per row and KS2 wherever KS2 cannot stream rows by TMA (L not a multiple of the
+    // vector): profiles/r02_scan_regimes_odd.jsonl (L = 8191: 0.57 -> 0.89, 65537: 0.75 -> 0.99)
+    const bool ring = op != FS_ARGMIN && al16;
     const bool ok[13] = {
         false, false, false, false, false,
         true,                                                                         // 5 look-back
@@ -1540,8 +1545,8 @@ int seg_scan_plan(int op, int dt, int64_t n, int64_t L, bool al16, bool co16, bo
     if (f >= 5 && f <= 12 && ok[f]) return f;
     if (ok[RG_KS0]) return RG_KS0;
     if (ok[RG_KS0_BIG]) return RG_KS0_BIG;
-    if (ok[RG_KS2]) return RG_KS2;
-    if (ok[RG_KS3]) return RG_KS3;
+    if (ok[RG_KS2] && (!ring || L % VEC == 0)) return RG_KS2;
+    if (ok[RG_KS3] && (!ring || L <= 4096)) return RG_KS3;
     if (ok[RG_KS1]) return RG_KS1;
     if (ok[RG_FLAT_ROW] && L >= kFlatRowMin) return RG_FLAT_ROW;
     return RG_KS_LOOKBACK;
@@ -1750,6 +1755,15 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
                     const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((j * kRingA + at) << 4)));
 #pragma unroll
                     for (int q = 0; q < VEC; ++q) acc = O::comb(acc, a.e[q]);
+                }
+            } else if (nv == TILE) {  // SEG, a start in the tile: the same vector loads, masked
+#pragma unroll
+                for (int j = 0; j < 2 * kRingVPT; ++j) {
+                    const int e = (j * kRingA + at) * VEC;
+                    const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((j * kRingA + at) << 4)));
+#pragma unroll
+                    for (int q = 0; q < VEC; ++q)
+                        if (e + q >= lo) acc = O::comb(acc, a.e[q]);
                 }
             } else {
                 for (int j = 0; j < 2 * kRingVPT; ++j) {

@@ -210,7 +210,7 @@ def test_workspace_queries_and_regimes(fs):
     assert r(64, 64, layout="col") == 4
     assert r(64, 64, scan=True) == 7 and r(1 << 20, 1024, scan=True) == 7 and r(64, 63, scan=True) == 11
     assert r(1 << 20, 3, scan=True) == 11 and r(1 << 20, 33, scan=True) == 11 and r(64, 7, scan=True, op="argmin") == 5
-    assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 11  # KS2: >= 1 row per SM
+    assert r(1 << 12, 16384, scan=True) == 9 and r(64, 16384, scan=True) == 5 and r(64, 4092, scan=True) == 11 and r(64, 4100, scan=True) == 5  # KS2: >= 1.7 x SMs rows; the ring above 4096
     assert r(64, 16384, scan=True, op="argmin") == 5 and r(64, 16385, scan=True) == 5
     assert r(1 << 12, 2048, scan=True) == 10 and r(1 << 12, 2048, scan=True, dtype=torch.int64) == 10
     assert r(1 << 12, 8192, scan=True) == 10 and r(1 << 12, 16384, scan=True, dtype=torch.int64) == 9
