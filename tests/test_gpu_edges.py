@@ -398,3 +398,21 @@ def test_seg_scan_ring_rows_around_tile(fs, dt):
                     eq(got, want, f"ring seg_scan {np.dtype(dt).name} {op} {nseg}x{L}")
     finally:
         fs.force_seg_regime(-1)
+
+
+# ------------------------------------------------------------------ long columns
+@pytest.mark.parametrize("nseg,seglen", [(4, 700_001), (8, 400_003), (16, 200_000), (32, 90_001), (64, 47_777),
+                                         (128, 23_333), (256, 12_001)])
+def test_seg_scan_col_long(fs, nseg, seglen):
+    """Column-major seg_scan of few long columns (the narrow and one-pass look-back column
+    kernels, ragged row blocks); int wrap-around, min/max bit-exact, f32 add within R2."""
+    for dt, op in ((np.float32, "add"), (np.int32, "add"), (np.int32, "max"), (np.float32, "min")):
+        x = workloads.full_range(nseg * seglen, nseg + seglen, dt) if (op == "add" and dt == np.int32) else \
+            workloads.mixed(nseg * seglen, nseg * 7 + seglen, dt)
+        got = fs.seg_scan(cu(x), nseg, seglen, op, layout="col")
+        want = oracle.seg_scan(x, nseg, seglen, op, "col")
+        if op == "add" and dt == np.float32:
+            asum = oracle.seg_scan(np.abs(x), nseg, seglen, "add", "col")
+            assert np.all(np.abs(host(got).astype(np.float64) - want) <= 1e-4 * asum + 1e-30), (nseg, seglen)
+        else:
+            eq(got, want, f"col long {nseg}x{seglen} {np.dtype(dt).name} {op}")

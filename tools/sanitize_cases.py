@@ -134,3 +134,18 @@ fs.seg_scan(xs[: 149 * 12_292], 149, 12_292, "add")
 fs.seg_scan(xs8[: 150 * 12_292], 150, 12_292, "min")
 torch.cuda.synchronize()
 print("sanitize cases done")
+# round 2: the ring scan (scanomap and the aligned segmented look-back): more tiles than CTAs
+# (every ring slot reused, both consumer groups, end markers), a ragged sub-vector tail, 8-byte
+# tiles, a carry-in, segment starts inside tiles (masked aggregate vectors)
+xg = cu(workloads.mixed(2_000_003, 17, np.float32))
+xg8 = cu(workloads.mixed(1_000_001, 18, np.int64))
+fs.scanomap(xg, "add")
+fs.scanomap(xg8, "max")
+fs.scanomap(xg[:777_777], "add", carry=xg[:1].clone())
+fs.force_seg_regime(5)
+fs.seg_scan(xg[: 100 * 10_001], 100, 10_001, "add")
+fs.seg_scan(xg8[: 300 * 3001], 300, 3001, "min")
+fs.force_seg_regime(-1)
+fs.seg_scan(xg[: 50 * 40_001], 50, 40_001, "max")  # the plan's ring choice (L > 4096, L % 4 != 0)
+torch.cuda.synchronize()
+print("ring cases ok")

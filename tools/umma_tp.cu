@@ -39,10 +39,10 @@ __global__ void tp(long long *out, int reps) {
     asm volatile("tcgen05.fence::after_thread_sync;");
     const uint32_t tm = tbase;
     if (t < 32) {  // one warp issues (elect lane 0 inside)
-        constexpr uint32_t id = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((128u >> 4) << 24);
+        constexpr uint32_t id = (1u << 4) | (1u << 7) | (1u << 10) | (MODE == 4 ? (1u << 15) : 0u) | ((uint32_t)(N >> 3) << 17) | ((128u >> 4) << 24);
         const uint32_t s0 = sa(sm);
-        const uint64_t a0 = (MODE == 0 || MODE == 2) ? desc(s0, 128, 256, 0) : desc(s0, 16, 1024, 2);
-        const uint64_t b0 = (MODE == 0 || MODE == 2) ? desc(s0 + 65536, 128, 256, 0) : desc(s0 + 65536, 16, 1024, 2);
+        const uint64_t a0 = MODE == 4 ? desc(s0, 1280, 128, 0) : ((MODE == 0 || MODE == 2) ? desc(s0, 128, 256, 0) : desc(s0, 16, 1024, 2));
+        const uint64_t b0 = MODE == 4 ? desc(s0 + 65536, 128, 2048, 0) : ((MODE == 0 || MODE == 2) ? desc(s0 + 65536, 128, 256, 0) : desc(s0 + 65536, 16, 1024, 2));
         long long best = 1ll << 60;
         for (int rep = 0; rep < reps; ++rep) {
             __syncwarp();
@@ -53,7 +53,7 @@ __global__ void tp(long long *out, int reps) {
                     constexpr int DC = 256 / NACC > N ? N : 256 / NACC;
                     const uint32_t dcol = tm + 256 + (uint32_t)((i % NACC) * DC);
                     const uint64_t off = (MODE == 1 || MODE == 3) ? (uint64_t)((i & 3) * 2) : 0;
-                    if (MODE < 2) mma_ss(dcol, a0 + off, b0 + off, id, i >= NACC);
+                    if (MODE < 2 || MODE == 4) mma_ss(dcol, a0 + (MODE == 4 ? (uint64_t)((i & 7) * 2 * 1280 >> 4) : off), b0 + (MODE == 4 ? (uint64_t)((i & 7) * 256 >> 4) : off), id, i >= NACC);
                     else mma_ts(dcol, tm + 8 * (i & 15), b0 + off, id, i >= NACC);
                 }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(sa(&bar)));
@@ -90,5 +90,6 @@ int main() {
     long long *d;
     cudaMalloc(&d, 8);
     runm<0>(d, "SS noswz"); runm<1>(d, "SS sw128"); runm<2>(d, "TS noswz"); runm<3>(d, "TS sw128");
+    runm<4>(d, "SS A-MN");
     return 0;
 }
