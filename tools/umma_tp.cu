@@ -86,10 +86,74 @@ template <int MODE> void runm(long long *d, const char *name) {
     run1<MODE, 64, 1>(d, name); run1<MODE, 64, 4>(d, name);
     run1<MODE, 128, 1>(d, name); run1<MODE, 128, 2>(d, name); run1<MODE, 256, 1>(d, name);
 }
+// the K-means stage mix: 5 MMA1 (A in TMEM, N = 64, K-major B) + 8 MMA2 (A MN-major, N = 32)
+__global__ void mix(long long *out, int reps) {
+    extern __shared__ __align__(1024) unsigned char sm[];
+    __shared__ uint64_t bar;
+    __shared__ uint32_t tbase;
+    const int t = threadIdx.x;
+    for (int e = t; e < 160 * 1024 / 4; e += blockDim.x) reinterpret_cast<float *>(sm)[e] = 0.f;
+    if (t < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(sa(&tbase)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (t == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sa(&bar)));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+    }
+    asm volatile("fence.proxy.async.shared::cta;");
+    asm volatile("tcgen05.fence::before_thread_sync;");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;");
+    const uint32_t tm = tbase;
+    if (t < 32) {
+        constexpr uint32_t id1 = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(64 >> 3) << 17) | ((128u >> 4) << 24);
+        constexpr uint32_t id2 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 15) | ((uint32_t)(32 >> 3) << 17) | ((128u >> 4) << 24);
+        const uint32_t s0 = sa(sm);
+        const uint64_t b1 = desc(s0 + 65536, 128, 1536, 0);
+        const uint64_t a2 = desc(s0, 1280, 128, 0), b2 = desc(s0 + 98304, 128, 2048, 0);
+        long long best = 1ll << 60;
+        for (int rep = 0; rep < reps; ++rep) {
+            __syncwarp();
+            const long long c0 = clock64();
+            if (t == 0) {
+#pragma unroll 1
+                for (int st = 0; st < 16; ++st) {
+#pragma unroll
+                    for (int p = 0; p < 5; ++p) mma_ts(tm + 64 * (st & 3), tm + 384 + 8 * p, b1 + (uint64_t)(p * 256 >> 4), id1, p > 0);
+#pragma unroll
+                    for (int kk = 0; kk < 8; ++kk)
+                        mma_ss(tm + 256 + 32 * (st & 1), a2 + (uint64_t)((kk * 2 * 1280) >> 4), b2 + (uint64_t)((kk * 256) >> 4), id2, 1);
+                }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(sa(&bar)));
+            }
+            __syncwarp();
+            uint32_t done = 0;
+            while (!done)
+                asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                             : "=r"(done) : "r"(sa(&bar)), "r"((unsigned)(rep & 1)));
+            const long long c1 = clock64();
+            if (c1 - c0 < best) best = c1 - c0;
+        }
+        if (t == 0) out[0] = best;
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;");
+    __syncthreads();
+    if (t < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tm));
+}
 int main() {
     long long *d;
     cudaMalloc(&d, 8);
     runm<0>(d, "SS noswz"); runm<1>(d, "SS sw128"); runm<2>(d, "TS noswz"); runm<3>(d, "TS sw128");
     runm<4>(d, "SS A-MN");
+    {
+        long long h;
+        cudaFuncSetAttribute(mix, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
+        mix<<<1, 128, 160 * 1024>>>(d, 8);
+        cudaError_t e = cudaDeviceSynchronize();
+        cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost);
+        printf("k-means stage mix (5 MMA1 TS N=64 + 8 MMA2 SS N=32): %.1f cycles per stage (%s)\n", h / 16.0,
+               cudaGetErrorString(e));
+    }
     return 0;
 }
