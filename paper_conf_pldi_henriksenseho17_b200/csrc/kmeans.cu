@@ -40,6 +40,7 @@
 //             f32 accumulation).
 // Chunk results combine CTA -> workspace -> last CTA, which divides by the counts.
 #include <cuda_bf16.h>
+#include <stdio.h>
 #include <stdlib.h>
 
 #include "internal.cuh"
@@ -167,6 +168,16 @@ __device__ __forceinline__ void tmem_st8u(uint32_t taddr, const uint32_t (&v)[8]
                  "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
                  : "memory");
 }
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const float (&v)[32]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+        "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]), "f"(v[8]), "f"(v[9]),
+        "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15]), "f"(v[16]), "f"(v[17]), "f"(v[18]),
+        "f"(v[19]), "f"(v[20]), "f"(v[21]), "f"(v[22]), "f"(v[23]), "f"(v[24]), "f"(v[25]), "f"(v[26]), "f"(v[27]),
+        "f"(v[28]), "f"(v[29]), "f"(v[30]), "f"(v[31])
+        : "memory");
+}
 __device__ __forceinline__ void tmem_st1(uint32_t taddr, float v) {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "r"(__float_as_uint(v)) : "memory");
 }
@@ -207,6 +218,8 @@ struct KmBars {
     uint32_t tmem_base;
     float cmax2;
     float nrm[kKmNA][kKmRows];  // |x|^2 of the rows of the stages in the TMEM slots
+    short ohpos[kKmNXMax][kKmRows];  // the one-hot entry row r set in X slot q (-1: none), reset
+                                     // by whichever decide group reuses the slot next
 };
 // running f32 totals of the D2 buffers ([128 M rows][NC]), after the barriers in shared memory
 
@@ -395,6 +408,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     }
     for (int e = tid; e < (int)((NX * (x2_bytes + oh_bytes) + 1024) / 16); e += kKmThreads)
         reinterpret_cast<uint4 *>(x2)[e] = make_uint4(0u, 0u, 0u, 0u);
+    for (int e = tid; e < kKmNXMax * kKmRows; e += kKmThreads) (&B.ohpos[0][0])[e] = -1;
     __syncthreads();
     // B1[n][k], K-major no swizzle: n < NC is centre n with the b1 piece of -2c and the |c|^2
     // pieces q1 q2 q3 in columns d, d+1, d+2 of the a1 half; n >= NC is centre n - NC with the b2
@@ -447,7 +461,10 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     tc_fence_after();
     const uint32_t tmem = B.tmem_base;
     // TMEM columns: D1 slots [0, NA N1), D2 buffers (2 NC), A slots (KP each): <= 4 64 + 64 + 4 48 = 512
-    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tA = tD2 + 2 * NC;
+    // A slots of KA columns: K1 / 2 with the packed layout (40 at d = 34), else KP; with the packed
+    // layout the D2 running totals take the 32 columns after the A slots (TMEM, not shared memory)
+    const int KA = PKD > 0 ? K1 / 2 : G.KP;
+    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tA = tD2 + 2 * NC, tT = tA + kKmNA * KA;
 
     float *s_part = reinterpret_cast<float *>(x2);  // [128][NC] CTA partial (after the loop)
     if (warp < kKmWarpDecide) {
@@ -473,7 +490,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             if (s >= kKmNA) km_wait(&B.slotfree[sa], (unsigned)(((s / kKmNA) - 1) & 1));  // decide read D1
             if (s >= NX) km_wait(&B.x2free[sx], (unsigned)(((s / NX) - 1) & 1));         // MMA2 read X
             tc_fence_after();
-            const uint32_t ta = tA + t_lane + (uint32_t)(sa * G.KP);
+            const uint32_t ta = tA + t_lane + (uint32_t)(sa * KA);
             unsigned char *xr = x2 + sx * x2_bytes + (r >> 3) * LB2 + (r & 7) * 16;
             KM_TRACE(s, 1);
             float nrm;
@@ -497,11 +514,17 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         const uint32_t t_lane = (uint32_t)(wl * 32) << 16;
         const float cmax2 = B.cmax2;
         float *acc_tot = s_acc + r;  // this thread's M row of the D2 totals (group 0): [c][128], conflict-free
-        if (dg == 0)
-            for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = 0.f;
-        int ohpos[kKmNXMax];
+        if (dg == 0) {
+            if constexpr (PKD > 0) {  // totals in TMEM lane r, columns tT..tT+31
+                float z[32];
 #pragma unroll
-        for (int q = 0; q < kKmNXMax; ++q) ohpos[q] = -1;
+                for (int c = 0; c < 32; ++c) z[c] = 0.f;
+                tmem_st32(tT + t_lane, z);
+                asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+            } else {
+                for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = 0.f;
+            }
+        }
         unsigned wdelta = 0;
         int flushed = 0;
         auto flush = [&]() {
@@ -510,8 +533,17 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             tc_fence_after();
             float v[32];
             tmem_ld32(tD2 + t_lane + (uint32_t)(b2 * NC), v);
+            if constexpr (PKD > 0) {
+                float tt[32];
+                tmem_ld32(tT + t_lane, tt);
 #pragma unroll
-            for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = __fadd_rn(acc_tot[c * kKmRows], v[c]);
+                for (int c = 0; c < NC; ++c) tt[c] = __fadd_rn(tt[c], v[c]);
+                tmem_st32(tT + t_lane, tt);
+                asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+            } else {
+#pragma unroll
+                for (int c = 0; c < NC; ++c) acc_tot[c * kKmRows] = __fadd_rn(acc_tot[c * kKmRows], v[c]);
+            }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) km_arrive(&B.d2free[b2]);
@@ -577,16 +609,11 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             // one-hot B operand of MMA2 (K-major bf16: [centre group][row chunk][8 x 16 B]); the
             // slot's previous MMA2 is complete (the convert of this stage waited for it)
             unsigned short *ohs = reinterpret_cast<unsigned short *>(oh + sx * oh_bytes);
-            int op = -1;
-#pragma unroll
-            for (int q = 0; q < kKmNXMax; ++q)
-                if (q == sx) op = ohpos[q];
+            int op = B.ohpos[sx][r];
             if (op >= 0) ohs[op] = 0;
             op = valid ? ((key >> 3) * 2048 + (r >> 3) * 128 + (key & 7) * 16 + (r & 7) * 2) / 2 : -1;
             if (valid) ohs[op] = 0x3F80;  // bf16 1.0
-#pragma unroll
-            for (int q = 0; q < kKmNXMax; ++q)
-                if (q == sx) ohpos[q] = op;
+            B.ohpos[sx][r] = (short)op;
             fence_proxy_async();
             __syncwarp();
             if (lane == 0) km_arrive(&B.ohfull[sx]);
@@ -604,8 +631,16 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         // every MMA has completed (the last D2 buffer follows every MMA2): the X slots may hold
         // the partial
         km_bar_sync(1, 4 * kKmDc * 32);
-        if (dg == 0)
-            for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c * kKmRows];
+        if (dg == 0) {
+            if constexpr (PKD > 0) {
+                float tt[32];
+                tmem_ld32(tT + t_lane, tt);
+#pragma unroll
+                for (int c = 0; c < NC; ++c) s_part[r * NC + c] = tt[c];
+            } else {
+                for (int c = 0; c < NC; ++c) s_part[r * NC + c] = acc_tot[c * kKmRows];
+            }
+        }
     } else if (warp == kKmWarpProd) {
         // =============================== producer: TMA bulk copies of full stages
         if (lane == 0) {
@@ -630,7 +665,7 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
                 km_wait(&B.a1full[sa], (unsigned)((s1 / kKmNA) & 1));  // (implies the D1 slot is free)
                 if (trace) trace[s1 * 16 + 8] = clock64();
                 tc_fence_after();
-                const uint32_t ta = tA + (uint32_t)(sa * G.KP), dt = tD1 + (uint32_t)(sa * N1);
+                const uint32_t ta = tA + (uint32_t)(sa * KA), dt = tD1 + (uint32_t)(sa * N1);
                 for (int p = 0; p < ((skip & 2) ? 0 : K1S); ++p)  // 8 TMEM columns (16 bf16) of A each
                     umma_bf16_ts(dt, ta + 8 * p, bdesc0 + (uint64_t)(p * 256 >> 4), id1, p > 0);
                 if (trace) trace[s1 * 16 + 9] = clock64();
@@ -727,20 +762,26 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     }
 }
 
-static size_t km_smem_bytes(int64_t d, int NC, int NR, int NX) {
+static size_t km_smem_bytes(int64_t d, int NC, int NR, int NX, bool pk) {
     const KmGeom G((int)d);
     const size_t raw_slot = align_up((size_t)kKmRows * d * 4, 1024);
     const size_t oh = (size_t)NC / 8 * 2048;
     const size_t b1 = (size_t)(2 * NC / 8) * (2 * G.KP / 8 * 128);
     return 1024 + NR * raw_slot + NX * ((size_t)G.x2_bytes() + oh) + 1024 + b1 + (size_t)NC * kKmMaxD * 4 +
-           sizeof(KmBars) + (size_t)kKmRows * NC * 4;
+           sizeof(KmBars) + (pk ? 0 : (size_t)kKmRows * NC * 4);  // (pk: the D2 totals live in TMEM)
 }
 // deepest rings that fit the 227 KB opt-in limit (+ the static shared words): X slots first
-static void km_rings(int64_t d, int NC, int &NR, int &NX) {
-    // NX even: a slot is always reused by the same decide group (it resets its own one-hot entries)
-    for (NX = kKmNXMax; NX >= 2; NX -= kKmDc)
+static void km_rings(int64_t d, int NC, bool pk, int &NR, int &NX) {
+    if (const char *e = getenv("FUTSEG_KM_RINGS")) {  // "NX,NR": ring-depth experiments
+        if (sscanf(e, "%d,%d", &NX, &NR) == 2 && NX >= 2 && NX <= kKmNXMax && NR >= 2 && NR <= kKmRing &&
+            km_smem_bytes(d, NC, NR, NX, pk) + 2048 <= 227 * 1024)
+            return;
+    }
+    // X slots first (the X-slot cycle convert -> MMA1 -> decide -> MMA2 is the critical loop),
+    // then raw slots (3 measured as fast as 4; 2 is slower)
+    for (NX = kKmNXMax; NX >= 2; --NX)
         for (NR = kKmRing; NR >= 3; --NR)
-            if (km_smem_bytes(d, NC, NR, NX) + 2048 <= 227 * 1024) return;
+            if (km_smem_bytes(d, NC, NR, NX, pk) + 2048 <= 227 * 1024) return;
     NR = 2;
     NX = 2;
 }
@@ -768,7 +809,8 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
     float *parts = (float *)(w + kWsHeader);
     int *pcnt = (int *)(w + kWsHeader + align_up((size_t)G * k * d * 4, 256));
     int NR, NX;
-    km_rings(d, NC, NR, NX);
+    constexpr bool pk = DT > 0 && DT % 2 == 0;
+    km_rings(d, NC, pk, NR, NX);
     {   // debug switches (tools/km_trace.py, tools/km_skip.py): set once per process and device,
         // only when requested (the device globals default to off: no copies on the product path)
         static const char *e = getenv("FUTSEG_KM_TRACE");
@@ -787,7 +829,7 @@ static fs_status km_launch(const float *pts, int64_t n, int d, const float *cen,
             done_dev |= 1u << dev;
         }
     }
-    const size_t smem = km_smem_bytes(d, NC, NR, NX);
+    const size_t smem = km_smem_bytes(d, NC, NR, NX, pk);
     auto kern = kmeans_tc_kernel<NC, DT>;
     cudaFuncSetAttribute((const void *)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     kern<<<(unsigned)G, kKmThreads, smem, st>>>(pts, n, d, NR, NX, cen, k, prev, membership, rows, parts, pcnt,
