@@ -486,8 +486,10 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             } else {
                 src = pts + (r0 + (valid ? r : 0)) * d;
             }
+            KM_TRACE(s, 12);
             const int sa = s % kKmNA, sx = s % NX;
             if (s >= kKmNA) km_wait(&B.slotfree[sa], (unsigned)(((s / kKmNA) - 1) & 1));  // decide read D1
+            KM_TRACE(s, 13);
             if (s >= NX) km_wait(&B.x2free[sx], (unsigned)(((s / NX) - 1) & 1));         // MMA2 read X
             tc_fence_after();
             const uint32_t ta = tA + t_lane + (uint32_t)(sa * KA);

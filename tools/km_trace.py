@@ -47,3 +47,6 @@ print("events per stage around a gap (cols: cv_begin cv_ready cv_end dc_begin dc
 base = t[g0 - 8, 0]
 for i in range(g0 - 8, g0 + 4):
     print(i + 5, (i + 5) % 16, [int(v - base) for v in t[i, :8]])
+# convert waits: raw slot (begin -> 12), TMEM slot (12 -> 13), X slot (13 -> ready)
+print("convert waits (median cycles): raw", np.median(t[:, 12] - t[:, 0]), " tmem slot", np.median(t[:, 13] - t[:, 12]),
+      " x slot", np.median(t[:, 1] - t[:, 13]))
