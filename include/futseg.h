@@ -143,8 +143,10 @@ fs_status fs_redomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *
  *   carry / carry_idx: optional DEVICE pointers to one element (and, for ARGMIN,
  *   one int64 index) folded in front of the scan: c.  NULL means c = 0(+).
  *   (Used to continue a scan across shards: F5's accumulator a.)
- * Single-pass chained scan with decoupled look-back; the workspace holds the
- * per-tile status words and is re-initialised by every call. */
+ * Single-pass chained scan with decoupled look-back (add/min/max on 16-byte aligned
+ * buffers: the ring scan, every tile held in shared memory between its read and its
+ * write); the workspace holds the per-tile status words and is re-initialised by every
+ * call. */
 fs_status fs_scanomap(fs_opdesc op, fs_mapdesc map, const void *in0, const void *in1, int64_t n,
                       void *out, int64_t *out_idx, const void *carry, const int64_t *carry_idx,
                       void *ws, size_t ws_bytes, void *stream);
