@@ -16,6 +16,8 @@
 //   KG4  L large, few segments  : C CTAs per segment; each writes a partial
 //                   and the last to arrive (per-segment ticket) combines the
 //                   C partials in chunk order (the "second pass", fused).
+#include <type_traits>
+
 #include "internal.cuh"
 
 namespace fs {
@@ -160,12 +162,39 @@ seg_rows_odd_kernel(const T *__restrict__ x, int64_t nseg, int L, T *out, int64_
 template <class O, typename T, int LS>
 __device__ __forceinline__ void small_segs(const Vec16<T> &e, int64_t v, T *out, int64_t *out_idx) {
     constexpr int VEC = 16 / sizeof(T), SPL = VEC / LS;
+    constexpr int OB = SPL * (int)sizeof(T);  // output bytes of one vector's segments
+    if constexpr (!std::is_same<typename O::V, T>::value || (OB != 8 && OB != 16)) {
 #pragma unroll
-    for (int sg = 0; sg < SPL; ++sg) {
-        typename O::V a = O::id();
+        for (int sg = 0; sg < SPL; ++sg) {
+            typename O::V a = O::id();
 #pragma unroll
-        for (int k = 0; k < LS; ++k) a = O::fold(a, e.e[sg * LS + k], k);
-        store_out<O>(out, out_idx, v * SPL + sg, a);
+            for (int k = 0; k < LS; ++k) a = O::fold(a, e.e[sg * LS + k], k);
+            store_out<O>(out, out_idx, v * SPL + sg, a);
+        }
+    } else {  // the SPL results leave as ONE 8- or 16-byte store (L = 1, 2: a copy-like stream)
+        T res[SPL];
+#pragma unroll
+        for (int sg = 0; sg < SPL; ++sg) {
+            typename O::V a = O::id();
+#pragma unroll
+            for (int k = 0; k < LS; ++k) a = O::fold(a, e.e[sg * LS + k], k);
+            res[sg] = a;
+        }
+        T *dst = out + v * SPL;
+        if (((uintptr_t)dst & (OB - 1)) == 0) {
+            if constexpr (OB == 16) {
+                int4 w;
+                memcpy(&w, res, 16);
+                *reinterpret_cast<int4 *>(dst) = w;
+            } else {
+                int2 w;
+                memcpy(&w, res, 8);
+                *reinterpret_cast<int2 *>(dst) = w;
+            }
+        } else {
+#pragma unroll
+            for (int sg = 0; sg < SPL; ++sg) dst[sg] = res[sg];
+        }
     }
 }
 
