@@ -344,7 +344,9 @@ static PeriodPlan period_plan(int dt, int op, int64_t m, int64_t w, int64_t resi
 // its m x 4 loads at once (scalar loads; a warp's loads of one row are 512 contiguous bytes, so
 // they coalesce whatever the row phase), then folds each column down the rows in order.  The
 // column-major seg_reduce of short segments (seglen = 3, 7: an elementwise combine of m rows).
-template <int OP, typename T, int MMAX>
+// VECIO (four-byte T, 16-byte aligned x and out, w % 4 == 0): every row's 4 columns arrive as
+// one 16-byte load and the 4 results leave as one 16-byte store.
+template <int OP, typename T, int MMAX, bool VECIO>
 __global__ void __launch_bounds__(256)
 colreduce_short_kernel(const T *__restrict__ x, int m, int64_t w, T *out, int64_t *out_idx) {
     using O = Op<OP, T>;
@@ -354,19 +356,41 @@ colreduce_short_kernel(const T *__restrict__ x, int m, int64_t w, T *out, int64_
     for (int64_t g = (int64_t)blockIdx.x * 256 + threadIdx.x; g < ng; g += (int64_t)gridDim.x * 256) {
         const int64_t c0 = g * C;
         T v[MMAX][C];
-#pragma unroll
-        for (int r = 0; r < MMAX; ++r)
-#pragma unroll
-            for (int k = 0; k < C; ++k)
-                if (r < m && c0 + k < w) v[r][k] = __ldg(x + (int64_t)r * w + c0 + k);
-#pragma unroll
-        for (int k = 0; k < C; ++k) {
-            if (c0 + k >= w) break;
-            V a = O::id();
+        if constexpr (VECIO) {
 #pragma unroll
             for (int r = 0; r < MMAX; ++r)
-                if (r < m) a = O::fold(a, v[r][k], r);
-            store_out<O>(out, out_idx, c0 + k, a);
+                if (r < m) {
+                    const Vec16<T> e = as_vec<T>(ldg16(x + (int64_t)r * w + c0));
+#pragma unroll
+                    for (int k = 0; k < C; ++k) v[r][k] = e.e[k];
+                }
+            Vec16<T> o;
+#pragma unroll
+            for (int k = 0; k < C; ++k) {
+                V a = O::id();
+#pragma unroll
+                for (int r = 0; r < MMAX; ++r)
+                    if (r < m) a = O::fold(a, v[r][k], r);
+                o.e[k] = O::val(a);
+            }
+            int4 ov;
+            memcpy(&ov, &o, 16);
+            *reinterpret_cast<int4 *>(out + c0) = ov;
+        } else {
+#pragma unroll
+            for (int r = 0; r < MMAX; ++r)
+#pragma unroll
+                for (int k = 0; k < C; ++k)
+                    if (r < m && c0 + k < w) v[r][k] = __ldg(x + (int64_t)r * w + c0 + k);
+#pragma unroll
+            for (int k = 0; k < C; ++k) {
+                if (c0 + k >= w) break;
+                V a = O::id();
+#pragma unroll
+                for (int r = 0; r < MMAX; ++r)
+                    if (r < m) a = O::fold(a, v[r][k], r);
+                store_out<O>(out, out_idx, c0 + k, a);
+            }
         }
     }
 }
@@ -417,12 +441,23 @@ template <int OP, typename T> struct ColRun {
         if (m <= 8 && w >= resident * 256) {  // few rows, many columns: elementwise, any alignment
             const int64_t ng = ceil_div(w, 4);
             const int64_t grid = ceil_div(ng, 256) < resident * 2 ? ceil_div(ng, 256) : resident * 2;
+            if constexpr (sizeof(T) == 4 && OP != kArgmin) {
+                if (aligned && ((uintptr_t)out & 15) == 0 && w % 4 == 0) {
+                    if (m <= 4)
+                        colreduce_short_kernel<OP, T, 4, true><<<(unsigned)grid, 256, 0, st>>>(
+                            (const T *)in, (int)m, w, (T *)out, out_idx);
+                    else
+                        colreduce_short_kernel<OP, T, 8, true><<<(unsigned)grid, 256, 0, st>>>(
+                            (const T *)in, (int)m, w, (T *)out, out_idx);
+                    return launch_status();
+                }
+            }
             if (m <= 4)
-                colreduce_short_kernel<OP, T, 4><<<(unsigned)grid, 256, 0, st>>>((const T *)in, (int)m, w, (T *)out,
-                                                                               out_idx);
+                colreduce_short_kernel<OP, T, 4, false><<<(unsigned)grid, 256, 0, st>>>((const T *)in, (int)m, w,
+                                                                                      (T *)out, out_idx);
             else
-                colreduce_short_kernel<OP, T, 8><<<(unsigned)grid, 256, 0, st>>>((const T *)in, (int)m, w, (T *)out,
-                                                                               out_idx);
+                colreduce_short_kernel<OP, T, 8, false><<<(unsigned)grid, 256, 0, st>>>((const T *)in, (int)m, w,
+                                                                                      (T *)out, out_idx);
             return launch_status();
         }
         char *wsb = (char *)ws;
