@@ -886,13 +886,18 @@ segscan_vec_kernel(const T *__restrict__ x, int64_t n, int L, int G, T *__restri
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t gid0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t iters = (nvec + stride - 1) / stride;  // warp-uniform: every lane shuffles
-    for (int64_t it0 = 0; it0 < iters; it0 += U) {
-        int4 r[U];
+    // software pipeline: the next batch's loads are in flight while this batch is scanned
+    int4 r[U], rn[U];
+    auto load_batch = [&](int64_t i0, int4 (&dst)[U]) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-            const int64_t v = gid0 + (it0 + u) * stride;
-            if (it0 + u < iters && v < nvec) r[u] = ldg16(x + v * VEC);
+            const int64_t v = gid0 + (i0 + u) * stride;
+            if (i0 + u < iters && v < nvec) dst[u] = ldg16(x + v * VEC);
         }
+    };
+    if (iters > 0) load_batch(0, r);
+    for (int64_t it0 = 0; it0 < iters; it0 += U) {
+        if (it0 + U < iters) load_batch(it0 + U, rn);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             const int64_t v = gid0 + (it0 + u) * stride;
@@ -931,6 +936,8 @@ segscan_vec_kernel(const T *__restrict__ x, int64_t n, int L, int G, T *__restri
                     for (int k = 0; k < VEC; ++k) out_idx[v * VEC + k] = O::idx(a[k]);
             }
         }
+#pragma unroll
+        for (int u = 0; u < U; ++u) r[u] = rn[u];
     }
     // ragged tail (L < VEC and n not a multiple of VEC): whole segments, one per thread
     const int64_t t0 = nvec * VEC;
