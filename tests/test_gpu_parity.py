@@ -185,6 +185,11 @@ def test_dirty_workspace_body(fs):
     np.testing.assert_array_equal(host(fs.scanomap(cu(x), "add")), oracle.scan(x, "add"))
     dirty()
     np.testing.assert_array_equal(host(fs.seg_reduce(cu(x), 3, 70_001, "max")), oracle.seg_reduce(x, 3, 70_001, "max"))
+    dirty()  # the ring scan's segmented look-back (status words zeroed per call, payload never)
+    np.testing.assert_array_equal(host(fs.seg_scan(cu(x), 3, 70_001, "add")), oracle.seg_scan(x, 3, 70_001, "add"))
+    x8 = workloads.full_range(333_333, 6, np.int64)
+    dirty()  # eight-byte tiles: status words plus separate aggregate / inclusive payload arrays
+    np.testing.assert_array_equal(host(fs.scanomap(cu(x8), "add")), oracle.scan(x8, "add"))
     dirty()
     s_, c_ = fs.stream_red(cu(pts), cu(prev), 32)
     np.testing.assert_array_equal(host(c_), oracle.stream_red(pts, prev, 32)[1])
