@@ -50,7 +50,10 @@ namespace fs {
 constexpr int kKmRows = 128;   // rows per stage (UMMA M)
 constexpr int kKmRing = 5;     // TMA ring slots (at most)
 constexpr int kKmCv = 2;       // convert groups of 4 warps; group g converts stages s = g (mod 2)
-constexpr int kKmNA = 4;       // TMEM stage slots (A operand, D1)
+#ifndef FS_KM_NA
+#define FS_KM_NA 4
+#endif
+constexpr int kKmNA = FS_KM_NA;  // TMEM stage slots (A operand, D1); 5 measured no faster than 4
 constexpr int kKmDc = 2;       // decide groups of 4 warps; group g decides stages s = g (mod 2)
 constexpr int kKmNXMax = 6;    // shared-memory stage slots (MMA2 operands), at most
 constexpr int kKmThreads = (4 * kKmCv + 4 * kKmDc + 3) * 32;  // convert + decide + producer + 2 MMA warps
@@ -460,11 +463,12 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = B.tmem_base;
-    // TMEM columns: D1 slots [0, NA N1), D2 buffers (2 NC), A slots (KP each): <= 4 64 + 64 + 4 48 = 512
+    // TMEM columns: D1 slots [0, NA NC) (both b pieces accumulate into the same NC columns), D2
+    // buffers (2 NC), A slots (KA each), D2 running totals (packed layout): 5 32 + 64 + 5 40 + 32 <= 512
     // A slots of KA columns: K1 / 2 with the packed layout (40 at d = 34), else KP; with the packed
     // layout the D2 running totals take the 32 columns after the A slots (TMEM, not shared memory)
     const int KA = PKD > 0 ? K1 / 2 : G.KP;
-    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * N1, tA = tD2 + 2 * NC, tT = tA + kKmNA * KA;
+    const uint32_t tD1 = tmem, tD2 = tmem + kKmNA * NC, tA = tD2 + 2 * NC, tT = tA + kKmNA * KA;
 
     float *s_part = reinterpret_cast<float *>(x2);  // [128][NC] CTA partial (after the loop)
     if (warp < kKmWarpDecide) {
@@ -563,18 +567,10 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
             tc_fence_after();
             float dd[NC];
             {
-                float v[32];
-                tmem_ld32(tD1 + t_lane + (uint32_t)(sa * N1), v);
+                float v[32];  // (NC = 16: the upper 16 columns belong to the next slot, unused)
+                tmem_ld32(tD1 + t_lane + (uint32_t)(sa * NC), v);
 #pragma unroll
                 for (int c = 0; c < NC; ++c) dd[c] = v[c];
-                if (NC == 32) {
-                    tmem_ld32(tD1 + t_lane + (uint32_t)(sa * N1 + 32), v);
-#pragma unroll
-                    for (int c = 0; c < NC; ++c) dd[c] = __fadd_rn(dd[c], v[c]);
-                } else {
-#pragma unroll
-                    for (int c = 0; c < NC; ++c) dd[c] = __fadd_rn(dd[c], v[NC + c]);
-                }
             }
             const float nrm = B.nrm[sa][r];
             KM_TRACE(s, 4);
@@ -656,20 +652,23 @@ kmeans_tc_kernel(const float *__restrict__ pts, int64_t n, int d_rt, int NR, int
         }
     } else {
         // =============================== MMA issuers: one thread for MMA1, one for MMA2
-        constexpr uint32_t id1 = umma_idesc_bf16(N1, 0, 0);
+        constexpr uint32_t id1 = umma_idesc_bf16(NC, 0, 0);  // N = NC: the b1 and b2 pieces in turn
         constexpr uint32_t id2 = umma_idesc_bf16(NC, 1, 0);  // A (X) MN-major, B (one-hot) K-major
         if (warp == kKmWarpMma && lane == 0) {
             const uint32_t b10 = km_smem(b1);
             const int K1S = K1 / 16;  // MMA1 instructions (K = 16 each)
-            const uint64_t bdesc0 = umma_desc(b10, 128, SB1);
+            const uint64_t bdesc0 = umma_desc(b10, 128, SB1);                     // b1 rows n < NC
+            const uint64_t bdesc1 = umma_desc(b10 + (uint32_t)(NC / 8) * SB1, 128, SB1);  // b2 rows
             for (int s1 = 0; s1 < ns; ++s1) {
                 const int sa = s1 % kKmNA;
                 km_wait(&B.a1full[sa], (unsigned)((s1 / kKmNA) & 1));  // (implies the D1 slot is free)
                 if (trace) trace[s1 * 16 + 8] = clock64();
                 tc_fence_after();
-                const uint32_t ta = tA + (uint32_t)(sa * KA), dt = tD1 + (uint32_t)(sa * N1);
-                for (int p = 0; p < ((skip & 2) ? 0 : K1S); ++p)  // 8 TMEM columns (16 bf16) of A each
+                const uint32_t ta = tA + (uint32_t)(sa * KA), dt = tD1 + (uint32_t)(sa * NC);
+                for (int p = 0; p < ((skip & 2) ? 0 : K1S); ++p) {  // 8 TMEM columns (16 bf16) of A each
                     umma_bf16_ts(dt, ta + 8 * p, bdesc0 + (uint64_t)(p * 256 >> 4), id1, p > 0);
+                    umma_bf16_ts(dt, ta + 8 * p, bdesc1 + (uint64_t)(p * 256 >> 4), id1, 1);
+                }
                 if (trace) trace[s1 * 16 + 9] = clock64();
                 umma_commit(&B.d1full[sa]);
                 if (trace) trace[s1 * 16 + 6] = clock64();
