@@ -123,6 +123,30 @@ template <class S> struct TileState<S, false> {
     }
 };
 
+// 8-byte values (ring scan): value and status in ONE 16-byte word, stored and loaded with single
+// 16-byte relaxed accesses (as CUB's tile state does), so a look-back step costs one L2 round
+// trip as with PACK.  The status half also carries a 29-bit check of the value: a read that saw
+// the new status with a stale value (were a 16-byte access ever split) fails the check and is
+// treated as not yet published.
+template <class S> struct TileStateW {
+    uint64_t *w;  // 2 words per tile
+    static __device__ __forceinline__ uint64_t chk(uint64_t v) {
+        return (uint64_t)(((uint32_t)(v ^ (v >> 32)) * 0x9E3779B1u) >> 3);
+    }
+    __device__ __forceinline__ void publish(int64_t t, S s, unsigned st) const {
+        const uint64_t lo = (uint64_t)s.v, hi = (chk(lo) << 3) | (s.f ? 4ull : 0ull) | st;
+        asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(w + 2 * t), "l"(lo), "l"(hi) : "memory");
+    }
+    __device__ __forceinline__ unsigned poll(int64_t t, S &s) const {
+        uint64_t lo, hi;
+        asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(w + 2 * t) : "memory");
+        unsigned st = (unsigned)(hi & 3);
+        if (st && (hi >> 3) != chk(lo)) st = 0;
+        s.v = (decltype(s.v))lo;
+        s.f = (int)((hi >> 2) & 1);
+        return st;
+    }
+};
 
 #ifndef FS_SCAN_R
 #define FS_SCAN_R 4
@@ -1610,12 +1634,15 @@ constexpr int kRingVPT = FS_RING_VPT, kRingStages = FS_RING_STAGES, kRingG = 256
 constexpr int kRingThreads = kRingNG * kRingG + kRingA + 32;
 static_assert(kRingVPT % 2 == 1, "odd vectors per thread: conflict-free 16-byte shared loads");
 template <int OP, typename T> struct RingShape {
-    static constexpr bool PACK = sizeof(T) == 4;
+    static constexpr bool PACK = sizeof(T) == 4;  // 8-byte values: TileStateW (16-byte words)
     static constexpr int VEC = 16 / sizeof(T), E = kRingVPT * VEC;
     static constexpr int64_t TILE = (int64_t)kRingG * E;
     static constexpr unsigned TILE_BYTES = kRingG * kRingVPT * 16;
     static constexpr unsigned SMEM = kRingStages * TILE_BYTES;
 };
+template <int OP, typename T, bool SEG>
+using RingState = typename std::conditional<RingShape<OP, T>::PACK, TileState<typename SOp<Op<OP, T>, SEG>::S, true>,
+                                            TileStateW<typename SOp<Op<OP, T>, SEG>::S>>::type;
 
 #ifdef FS_RING_TRACE
 // per-tile event times (%globaltimer, ns): issued, landed, aggregate published, prefix
@@ -1638,8 +1665,7 @@ extern "C" int fs_debug_ring_trace(void *host, size_t bytes) {
 template <int OP, typename T, bool SEG>
 __global__ void __launch_bounds__(kRingThreads, 1)
 scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__ out, const T *carry,
-                 unsigned *counter, TileState<typename SOp<Op<OP, T>, SEG>::S, RingShape<OP, T>::PACK> ts,
-                 int64_t ntiles) {
+                 unsigned *counter, RingState<OP, T, SEG> ts, int64_t ntiles) {
     using O = Op<OP, T>;
     using SO = SOp<O, SEG>;
     using S = typename SO::S;
@@ -2018,13 +2044,11 @@ template <int OP, typename T> struct ScanRun {
             if (!scan_ring_disabled()) {
                 using ShR = RingShape<OP, T>;
                 const int64_t ntr = ceil_div(n, ShR::TILE);
-                if (cudaMemsetAsync(counter, 0, 256 + scan_state_bytes(ntr), st) != cudaSuccess) return FS_ERR_CUDA;
-                TileState<S, ShR::PACK> tr;
+                // state words: 8 B per tile (PACK) or 16 B (TileStateW), zeroed per call
+                const size_t stb = ShR::PACK ? scan_state_bytes(ntr) : 2 * scan_state_bytes(ntr);
+                if (cudaMemsetAsync(counter, 0, 256 + stb, st) != cudaSuccess) return FS_ERR_CUDA;
+                RingState<OP, T, SEG> tr;
                 tr.w = ts.w;
-                if constexpr (!ShR::PACK) {
-                    tr.aggs = ts.aggs;
-                    tr.incls = ts.incls;
-                }
                 auto kr = scan_ring_kernel<OP, T, SEG>;
                 static bool attr = false;
                 if (!attr) {
