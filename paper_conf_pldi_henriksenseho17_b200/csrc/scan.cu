@@ -147,6 +147,33 @@ template <class S> struct TileStateW {
         return st;
     }
 };
+// ARGMIN with 4-byte values (slab scan): value, index and status in ONE 16-byte word, like
+// TileStateW: lo = value bits | (index + 1) bits 0..31 << 32, hi = (index + 1) bits 32..39 |
+// flag << 8 | status << 9 | a 53-bit check of the rest.  Indices below 2^40 - 1.
+template <class S> struct TileStateA {
+    uint64_t *w;  // 2 words per tile
+    static __device__ __forceinline__ uint64_t chk(uint64_t lo, uint64_t hb) {
+        const uint64_t h = (lo ^ (hb << 40)) * 0x9E3779B97F4A7C15ull;
+        return h >> 11;
+    }
+    __device__ __forceinline__ void publish(int64_t t, S s, unsigned st) const {
+        const uint64_t ip = (uint64_t)(s.v.i + 1);
+        const uint64_t lo = (uint64_t)to_bits(s.v.v) | (ip << 32), hb = (ip >> 32) & 0xFF;
+        const uint64_t hi = hb | (s.f ? 256ull : 0ull) | ((uint64_t)st << 9) | (chk(lo, hb) << 11);
+        asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(w + 2 * t), "l"(lo), "l"(hi) : "memory");
+    }
+    __device__ __forceinline__ unsigned poll(int64_t t, S &s) const {
+        uint64_t lo, hi;
+        asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(w + 2 * t) : "memory");
+        const uint64_t hb = hi & 0xFF;
+        unsigned st = (unsigned)((hi >> 9) & 3);
+        if (st && (hi >> 11) != chk(lo, hb)) st = 0;
+        s.v.v = from_bits<decltype(s.v.v)>((uint32_t)lo);
+        s.v.i = (int64_t)((lo >> 32) | (hb << 32)) - 1;
+        s.f = (int)((hi >> 8) & 1);
+        return st;
+    }
+};
 
 #ifndef FS_SCAN_R
 #define FS_SCAN_R 4
@@ -484,6 +511,11 @@ template <int OP, typename T> struct ScanWShape {
     static constexpr int STA = FS_SCANW_STA, STC = FS_SCANW_STC;
     static constexpr unsigned SMEM = (STA + STC) * TILE_BYTES;
 };
+template <int OP, typename T, bool SEG>
+using WsState = typename std::conditional<
+    ScanWShape<OP, T>::PACK, TileState<typename SOp<Op<OP, T>, SEG>::S, true>,
+    typename std::conditional<OP == kArgmin && sizeof(T) == 4, TileStateA<typename SOp<Op<OP, T>, SEG>::S>,
+                              TileState<typename SOp<Op<OP, T>, SEG>::S, false>>::type>::type;
 
 __device__ __forceinline__ void named_bar(int id, int count) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
@@ -534,7 +566,7 @@ template <int OP, typename T, bool SEG>
 __global__ void __launch_bounds__(kScanWThreads, 1)
 scan_ws_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
                int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx,
-               TileState<typename SOp<Op<OP, T>, SEG>::S, ScanWShape<OP, T>::PACK> ts, int64_t ntiles, int tps) {
+               WsState<OP, T, SEG> ts, int64_t ntiles, int tps) {
     using O = Op<OP, T>;
     using V = typename O::V;
     using SO = SOp<O, SEG>;
@@ -2074,8 +2106,17 @@ template <int OP, typename T> struct ScanRun {
                 const int64_t G = nslabs < G0 ? nslabs : G0;
                 auto kw = scan_ws_kernel<OP, T, SEG>;
                 cudaFuncSetAttribute((const void *)kw, cudaFuncAttributeMaxDynamicSharedMemorySize, ShW::SMEM);
+                WsState<OP, T, SEG> tw;
+                tw.w = ts.w;
+                if constexpr (!ShW::PACK && !(OP == kArgmin && sizeof(T) == 4)) {
+                    tw.aggs = ts.aggs;
+                    tw.incls = ts.incls;
+                }
+                if constexpr (OP == kArgmin && sizeof(T) == 4) {  // 16 B per slab tile, zeroed
+                    if (cudaMemsetAsync(ts.w, 0, 2 * scan_state_bytes(ntw), st) != cudaSuccess) return FS_ERR_CUDA;
+                }
                 kw<<<(unsigned)G, kScanWThreads, ShW::SMEM, st>>>((const T *)in0, n, L, map.ibase, (T *)out, out_idx,
-                                                                  (const T *)carry, carry_idx, ts, ntw, (int)tps);
+                                                                  (const T *)carry, carry_idx, tw, ntw, (int)tps);
                 return launch_status();
             }
         }
