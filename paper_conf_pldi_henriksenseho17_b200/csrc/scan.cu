@@ -1666,15 +1666,17 @@ constexpr int kRingVPT = FS_RING_VPT, kRingStages = FS_RING_STAGES, kRingG = 256
 constexpr int kRingThreads = kRingNG * kRingG + kRingA + 32;
 static_assert(kRingVPT % 2 == 1, "odd vectors per thread: conflict-free 16-byte shared loads");
 template <int OP, typename T> struct RingShape {
-    static constexpr bool PACK = sizeof(T) == 4;  // 8-byte values: TileStateW (16-byte words)
+    static constexpr bool PACK = sizeof(T) == 4 && OP != kArgmin;  // else 16-byte words (TileStateW / A)
     static constexpr int VEC = 16 / sizeof(T), E = kRingVPT * VEC;
     static constexpr int64_t TILE = (int64_t)kRingG * E;
     static constexpr unsigned TILE_BYTES = kRingG * kRingVPT * 16;
     static constexpr unsigned SMEM = kRingStages * TILE_BYTES;
 };
 template <int OP, typename T, bool SEG>
-using RingState = typename std::conditional<RingShape<OP, T>::PACK, TileState<typename SOp<Op<OP, T>, SEG>::S, true>,
-                                            TileStateW<typename SOp<Op<OP, T>, SEG>::S>>::type;
+using RingState = typename std::conditional<
+    OP == kArgmin, TileStateA<typename SOp<Op<OP, T>, SEG>::S>,
+    typename std::conditional<RingShape<OP, T>::PACK, TileState<typename SOp<Op<OP, T>, SEG>::S, true>,
+                              TileStateW<typename SOp<Op<OP, T>, SEG>::S>>::type>::type;
 
 #ifdef FS_RING_TRACE
 // per-tile event times (%globaltimer, ns): issued, landed, aggregate published, prefix
@@ -1696,8 +1698,11 @@ extern "C" int fs_debug_ring_trace(void *host, size_t bytes) {
 
 template <int OP, typename T, bool SEG>
 __global__ void __launch_bounds__(kRingThreads, 1)
-scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__ out, const T *carry,
-                 unsigned *counter, RingState<OP, T, SEG> ts, int64_t ntiles) {
+scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, int64_t ibase, T *__restrict__ out,
+                 int64_t *__restrict__ out_idx, const T *carry, const int64_t *carry_idx, unsigned *counter,
+                 RingState<OP, T, SEG> ts, int64_t ntiles) {
+    // ARGMIN: an element's index is its offset in its row (SEG) or ibase + its position (flat);
+    // out_idx receives the index of every prefix's minimum (16-byte aligned)
     using O = Op<OP, T>;
     using SO = SOp<O, SEG>;
     using S = typename SO::S;
@@ -1813,13 +1818,18 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
                     f = 1;
                 }
             }
+            // ARGMIN: index of tile element p = ib + p (no start at or before p in the tile: ib =
+            // the tile start's offset in its row, or ibase + t0 when flat) or p - lo (after the last start)
+            int64_t ib = 0;
+            if constexpr (OP == kArgmin) ib = SEG ? (f ? -lo : t0 % L) : ibase + t0;
             typename O::V acc = O::id();
             if (nv == TILE && lo == 0) {
 #pragma unroll
                 for (int j = 0; j < 2 * kRingVPT; ++j) {
+                    const int e = (j * kRingA + at) * VEC;
                     const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((j * kRingA + at) << 4)));
 #pragma unroll
-                    for (int q = 0; q < VEC; ++q) acc = O::comb(acc, a.e[q]);
+                    for (int q = 0; q < VEC; ++q) acc = O::comb(acc, O::lift(a.e[q], ib + e + q));
                 }
             } else if (nv == TILE) {  // SEG, a start in the tile: the same vector loads, masked
 #pragma unroll
@@ -1828,7 +1838,7 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
                     const Vec16<T> a = as_vec<T>(*reinterpret_cast<const int4 *>(slot + ((j * kRingA + at) << 4)));
 #pragma unroll
                     for (int q = 0; q < VEC; ++q)
-                        if (e + q >= lo) acc = O::comb(acc, a.e[q]);
+                        if (e + q >= lo) acc = O::comb(acc, O::lift(a.e[q], ib + e + q));
                 }
             } else {
                 for (int j = 0; j < 2 * kRingVPT; ++j) {
@@ -1837,7 +1847,8 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
                     for (int q = 0; q < VEC; ++q) {
                         const int64_t p = e + q;
                         if (p >= lo && p < nv)
-                            acc = O::comb(acc, p < nbulk ? reinterpret_cast<const T *>(slot)[p] : in[t0 + p]);
+                            acc = O::comb(acc, O::lift(p < nbulk ? reinterpret_cast<const T *>(slot)[p] : in[t0 + p],
+                                                       ib + p));
                     }
                 }
             }
@@ -1882,23 +1893,25 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
 #pragma unroll
             for (int i = 0; i < E; ++i) {
                 const int64_t p = e0 + i;
-                x[i] = p < nbulk ? reinterpret_cast<const T *>(slot)[p] : (p < nv ? in[t0 + p] : O::id());
+                x[i] = p < nbulk ? reinterpret_cast<const T *>(slot)[p] : (p < nv ? in[t0 + p] : O::val(O::id()));
             }
         }
         int64_t r0 = 0;
         if constexpr (SEG) r0 = (t0 + e0) % L;
         // no segment start among this thread's elements: the plain scan (flag 0)
         const bool noflag = !SEG || (r0 != 0 && L - r0 >= E);
+        // ARGMIN index of the thread's element i: xb + i (noflag or flat), else its row offset r
+        const int64_t xb = SEG ? r0 : ibase + t0 + e0;
         S run = SO::id();
         if (noflag) {
 #pragma unroll
-            for (int i = 0; i < E; ++i) run.v = O::comb(run.v, x[i]);
+            for (int i = 0; i < E; ++i) run.v = O::fold(run.v, x[i], xb + i);
         } else {
             int64_t r = r0;
 #pragma unroll
             for (int i = 0; i < E; ++i) {
                 S e;
-                e.v = x[i];
+                e.v = O::lift(x[i], r);
                 e.f = SEG ? (r == 0) : 0;
                 if (SEG) {
                     ++r;
@@ -1931,7 +1944,7 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
             // decoupled look-back over the published predecessors
             S exc = SO::id();
             if (t == 0) {
-                if (carry) exc = S{O::lift(*carry, -1), 0};
+                if (carry) exc = S{O::lift(*carry, carry_idx ? *carry_idx : -1), 0};
             } else {
                     // wide look-back: lane i polls predecessors j - EPL*i - 0 .. EPL-1 (all loads of a
                     // step in flight together: 32*EPL predecessors per L2 round trip)
@@ -1991,12 +2004,32 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
         }
         named_bar(1 + g, kRingG);
         const S p = SO::comb(s_wpre[g][warp], tex);
+        // ARGMIN: the prefix minima's indices leave as they are produced, two per 16-byte store
+        int64_t *oi = OP == kArgmin ? out_idx + t0 + e0 : nullptr;
+        int64_t pend = 0;
+        auto emit = [&](int i, int64_t idx) {
+            if constexpr (OP == kArgmin) {
+                if (nv == TILE) {
+                    if (i & 1) {
+                        longlong2 v2;
+                        v2.x = pend;
+                        v2.y = idx;
+                        *reinterpret_cast<longlong2 *>(oi + i - 1) = v2;
+                    } else {
+                        pend = idx;
+                    }
+                } else if (e0 + i < nv) {
+                    oi[i] = idx;
+                }
+            }
+        };
         if (noflag) {
             typename O::V c = p.v;
 #pragma unroll
             for (int i = 0; i < E; ++i) {
-                c = O::comb(c, x[i]);
+                c = O::comb(c, O::lift(x[i], xb + i));
                 x[i] = O::val(c);
+                emit(i, O::idx(c));
             }
         } else {
             S c = p;
@@ -2004,7 +2037,7 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
 #pragma unroll
             for (int i = 0; i < E; ++i) {
                 S e;
-                e.v = x[i];
+                e.v = O::lift(x[i], r);
                 e.f = SEG ? (r == 0) : 0;
                 if (SEG) {
                     ++r;
@@ -2012,6 +2045,7 @@ scan_ring_kernel(const T *__restrict__ in, int64_t n, int64_t L, T *__restrict__
                 }
                 c = SO::comb(c, e);
                 x[i] = O::val(c.v);
+                emit(i, O::idx(c.v));
             }
         }
         if (nv == TILE) {
@@ -2072,8 +2106,8 @@ template <int OP, typename T> struct ScanRun {
             ts.aggs = (S *)(b + 256 + scan_state_bytes(ntiles));
             ts.incls = ts.aggs + ntiles;
         }
-        if constexpr (TMA && !NN && OP != kArgmin) {  // the ring scan (16-byte aligned buffers)
-            if (!scan_ring_disabled()) {
+        if constexpr (TMA && !NN && (OP != kArgmin || sizeof(T) == 4)) {  // the ring scan (16-byte aligned)
+            if (!scan_ring_disabled() && (OP != kArgmin || ((uintptr_t)out_idx & 15) == 0)) {
                 using ShR = RingShape<OP, T>;
                 const int64_t ntr = ceil_div(n, ShR::TILE);
                 // state words: 8 B per tile (PACK) or 16 B (TileStateW), zeroed per call
@@ -2089,8 +2123,9 @@ template <int OP, typename T> struct ScanRun {
                 }
                 const int64_t G0 = sm_count();
                 const int64_t G = ntr < G0 ? ntr : G0;
-                kr<<<(unsigned)(G > 0 ? G : 1), kRingThreads, ShR::SMEM, st>>>((const T *)in0, n, L, (T *)out,
-                                                                               (const T *)carry, counter, tr, ntr);
+                kr<<<(unsigned)(G > 0 ? G : 1), kRingThreads, ShR::SMEM, st>>>((const T *)in0, n, L, map.ibase,
+                                                                               (T *)out, out_idx, (const T *)carry,
+                                                                               carry_idx, counter, tr, ntr);
                 return launch_status();
             }
         }
