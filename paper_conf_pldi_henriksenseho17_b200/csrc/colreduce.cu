@@ -421,7 +421,11 @@ static ColPlan col_plan(int dt, int64_t m, int64_t w, bool aligned, int op, int6
     // (tile, group) tickets + per-tile tickets of the two-level combine must fit too
     while (Y > 1 && p.tiles * (ceil_div(Y, kColGroup) + 1) > kWsMaxTickets) Y /= 2;
     const int64_t by_rows = m / ((int64_t)RB * 16);
-    const int64_t by_bytes = (m * (int64_t)dtype_size(dt)) / (100 * (int64_t)acc_size(op, dt));
+    // partial rows below ~1% of the input bytes -- ~4% for ARGMIN, whose 16-byte (value, index)
+    // partials would otherwise cap the row splits at a quarter and leave most of the GPU idle
+    // (col-major argmin L = 1024: 2 splits, 0.37 of HBM)
+    const int64_t by_bytes = (m * (int64_t)dtype_size(dt)) / (100 * (int64_t)(op == FS_ARGMIN ? dtype_size(dt)
+                                                                                             : acc_size(op, dt)));
     if (Y > by_rows) Y = by_rows;
     if (Y > by_bytes) Y = by_bytes;
     if (Y > 65535) Y = 65535;
