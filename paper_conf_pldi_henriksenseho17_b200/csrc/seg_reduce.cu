@@ -509,6 +509,16 @@ template <int OP, typename T> struct SegRun {
                                                                                             (T *)out, out_idx);
             return launch_status();
         }
+        if (regime == 0 && L == 2 * VEC && ((uintptr_t)x & 15) == 0) {  // one 32-byte segment per lane
+            const void *k = (const void *)seg_vecw_kernel<OP, T, kSegThreads, 2, 2>;
+            const int64_t nrun = nseg;
+            int64_t grid = ceil_div(nrun > 0 ? nrun : 1, (int64_t)kSegThreads * 2);
+            const int64_t cap = resident_blocks(k, kSegThreads);
+            grid = grid < cap ? grid : cap;
+            seg_vecw_kernel<OP, T, kSegThreads, 2, 2><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, 1,
+                                                                                         (T *)out, out_idx);
+            return launch_status();
+        }
         if (regime == 0 && pow2 && L <= 32 * VEC && ((uintptr_t)x & 15) == 0) {
             const int G = L > VEC ? (int)(L / VEC) : 1;
             const void *k = (const void *)seg_vec_kernel<OP, T, kSegThreads, 4>;
