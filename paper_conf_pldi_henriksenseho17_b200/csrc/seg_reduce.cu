@@ -490,6 +490,11 @@ static BlockPlan block_plan(int dt, int64_t nseg, int64_t L, int regime) {
     return p;
 }
 
+#ifndef FS_SEG_UPL
+// 16-byte vectors per lane run in KG0's wide-lane kernel: 2 (32-byte runs) measured 0.92-0.95 of
+// HBM for L = 8..256 f32, 4 (64-byte runs) 0.80-0.87 (profiles/r02_seg_upl.txt)
+#define FS_SEG_UPL 2
+#endif
 template <int OP, typename T> struct SegRun {
     static fs_status run(int regime, const void *in, int64_t nseg, int64_t L, void *out, int64_t *out_idx,
                          void *ws, cudaStream_t st) {
@@ -497,7 +502,7 @@ template <int OP, typename T> struct SegRun {
         const T *x = (const T *)in;
         constexpr int VEC = 16 / sizeof(T);
         const bool pow2 = (L & (L - 1)) == 0;
-        constexpr int UPL = 4;
+        constexpr int UPL = FS_SEG_UPL;
         if (regime == 0 && pow2 && L >= UPL * VEC && L <= 32 * UPL * VEC && ((uintptr_t)x & 15) == 0) {
             const int G = (int)(L / (UPL * VEC));
             const void *k = (const void *)seg_vecw_kernel<OP, T, kSegThreads, 2, UPL>;
@@ -507,16 +512,6 @@ template <int OP, typename T> struct SegRun {
             grid = grid < cap ? grid : cap;
             seg_vecw_kernel<OP, T, kSegThreads, 2, UPL><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, G,
                                                                                             (T *)out, out_idx);
-            return launch_status();
-        }
-        if (regime == 0 && L == 2 * VEC && ((uintptr_t)x & 15) == 0) {  // one 32-byte segment per lane
-            const void *k = (const void *)seg_vecw_kernel<OP, T, kSegThreads, 2, 2>;
-            const int64_t nrun = nseg;
-            int64_t grid = ceil_div(nrun > 0 ? nrun : 1, (int64_t)kSegThreads * 2);
-            const int64_t cap = resident_blocks(k, kSegThreads);
-            grid = grid < cap ? grid : cap;
-            seg_vecw_kernel<OP, T, kSegThreads, 2, 2><<<(unsigned)grid, kSegThreads, 0, st>>>(x, nseg, (int)L, 1,
-                                                                                         (T *)out, out_idx);
             return launch_status();
         }
         if (regime == 0 && pow2 && L <= 32 * VEC && ((uintptr_t)x & 15) == 0) {
