@@ -319,7 +319,7 @@ fs_status fs_check_device_error(void *ws, void *stream);
  *       16-byte loads (KG0), others thread/group per segment over a shared-memory
  *       tile (KG1)                                                     fs_seg_reduce
  *   1 = KG2 warp per segment                                            fs_seg_reduce
- *   2 = KG3 block per segment                                           fs_seg_reduce
+ *   2 = KG3 block per segment (at least 3 x SMs segments)              fs_seg_reduce
  *   3 = KG4 several blocks per segment, partials combined by the last   fs_seg_reduce
  *   4 = column kernels (FS_COL_MAJOR with nseg > 1 and seglen > 1)      both
  *   5 = single-pass segmented decoupled-look-back scan (the general case: argmin,

@@ -466,7 +466,10 @@ int seg_reduce_regime(int op, int dt, int64_t nseg, int64_t L) {
     if (L <= 64 || ((L & (L - 1)) == 0 && L <= 4 * 32 * vec / 2)) return 0;  // KG1 (KG0 when L is a power of two)
     if (L <= kWarpMaxL) return 1;
     const int64_t resident = (int64_t)sm_count() * 8;
-    return nseg >= 2 * resident ? 2 : 3;
+    // KG3 (a CTA per row) from 3 x SMs rows: the C4 sweep, 2^28 f32 (profiles/r02_kg34.txt), KG3 vs KG4:
+    // 4096 rows 0.95 / 0.90, 1024 0.94 / 0.89, 512 0.96 / 0.89, 256 0.80 / 0.92 (idle SMs)
+    (void)resident;
+    return nseg >= 3 * (int64_t)sm_count() ? 2 : 3;
 }
 
 struct BlockPlan {
