@@ -352,6 +352,31 @@ colreduce_short_kernel(const T *__restrict__ x, int m, int64_t w, T *out, int64_
     using O = Op<OP, T>;
     using V = typename O::V;
     constexpr int C = 4;
+    if constexpr (!VECIO) {
+        // any row phase: a warp takes 32 x C consecutive columns, lane-interleaved (column
+        // cw + lane + 32 k), so every load and store instruction touches 32 consecutive elements
+        const int lane = threadIdx.x & 31;
+        const int64_t nwb = (w + 32 * C - 1) / (32 * C);
+        for (int64_t b = ((int64_t)blockIdx.x * 256 + threadIdx.x) >> 5; b < nwb; b += ((int64_t)gridDim.x * 256) >> 5) {
+            const int64_t cw = b * 32 * C;
+            T v[MMAX][C];
+#pragma unroll
+            for (int r = 0; r < MMAX; ++r)
+#pragma unroll
+                for (int k = 0; k < C; ++k)
+                    if (r < m && cw + lane + 32 * k < w) v[r][k] = __ldg(x + (int64_t)r * w + cw + lane + 32 * k);
+#pragma unroll
+            for (int k = 0; k < C; ++k) {
+                if (cw + lane + 32 * k >= w) continue;
+                V a = O::id();
+#pragma unroll
+                for (int r = 0; r < MMAX; ++r)
+                    if (r < m) a = O::fold(a, v[r][k], r);
+                store_out<O>(out, out_idx, cw + lane + 32 * k, a);
+            }
+        }
+        return;
+    }
     const int64_t ng = (w + C - 1) / C;
     for (int64_t g = (int64_t)blockIdx.x * 256 + threadIdx.x; g < ng; g += (int64_t)gridDim.x * 256) {
         const int64_t c0 = g * C;
