@@ -2826,7 +2826,9 @@ template <int OP, typename T> struct ColScanRun {
     static fs_status run(const void *in, int64_t m, int64_t w, void *out, int64_t *out_idx, void *ws, cudaStream_t st) {
         const bool aligned = ((uintptr_t)in & 15) == 0 && ((uintptr_t)out & 15) == 0;
         const bool vec_ok = aligned && w % (16 / sizeof(T)) == 0;
-        if (m <= 8 && !vec_ok && w >= (int64_t)sm_count() * 2048) {  // few rows, many columns, any phase
+        // few rows, many columns: the lane-interleaved short kernel for any phase, and for aligned
+        // rows up to 2 (col L = 2: 0.70 -> 0.91; at 4 and 8 rows the vector kernels are faster)
+        if (m <= 8 && (!vec_ok || m <= 2) && w >= (int64_t)sm_count() * 2048) {
             const int64_t ng = ceil_div(w, 4 * 256);
             const int64_t gmax = (int64_t)sm_count() * 16;
             const unsigned grid = (unsigned)(ng < gmax ? ng : gmax);
