@@ -361,10 +361,20 @@ seg_warp_kernel(const T *__restrict__ x, int64_t nseg, int64_t L, T *out, int64_
                 for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], b + k);
             }
         }
-        for (; v < nvec; v += 32) {
-            const Vec16<T> e = as_vec<T>(ldg16(pv + v));
+        // the last partial batch: its (at most U) guarded loads issued together, one round trip
+        if (v < nvec) {
+            int4 r[U];
 #pragma unroll
-            for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], head + v * VEC + k);
+            for (int u = 0; u < U; ++u)
+                if (v + u * 32 < nvec) r[u] = ldg16(pv + v + u * 32);
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (v + u * 32 < nvec) {
+                    const Vec16<T> e = as_vec<T>(r[u]);
+                    const int64_t b = head + (v + u * 32) * VEC;
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k) a = O::fold(a, e.e[k], b + k);
+                }
         }
         if (lane < L - tail0) a = O::fold(a, __ldg(p + tail0 + lane), tail0 + lane);
         a = group_reduce<O>(a);
