@@ -148,10 +148,18 @@ colreduce_kernel(const T *__restrict__ x, int64_t m, int64_t w, int CG, int64_t 
                     for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], e.e[k], r + (int64_t)u * RB);
                 }
             }
-            for (; r < r1; r += RB) {
-                const Vec16<T> e = as_vec<T>(ldg16(base + r * w));
+            if (r < r1) {  // the last partial batch: guarded loads issued together
+                int4 v[U];
 #pragma unroll
-                for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], e.e[k], r);
+                for (int u = 0; u < U; ++u)
+                    if (r + (int64_t)u * RB < r1) v[u] = ldg16(base + (r + (int64_t)u * RB) * w);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (r + (int64_t)u * RB < r1) {
+                        const Vec16<T> e = as_vec<T>(v[u]);
+#pragma unroll
+                        for (int k = 0; k < VEC; ++k) acc[k] = O::fold(acc[k], e.e[k], r + (int64_t)u * RB);
+                    }
             }
         } else {
             for (; r + (int64_t)(U - 1) * RB < r1; r += (int64_t)U * RB) {
@@ -161,7 +169,15 @@ colreduce_kernel(const T *__restrict__ x, int64_t m, int64_t w, int CG, int64_t 
 #pragma unroll
                 for (int u = 0; u < U; ++u) acc[0] = O::fold(acc[0], v[u], r + (int64_t)u * RB);
             }
-            for (; r < r1; r += RB) acc[0] = O::fold(acc[0], __ldg(base + r * w), r);
+            if (r < r1) {  // the last partial batch: guarded loads issued together
+                T v[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (r + (int64_t)u * RB < r1) v[u] = __ldg(base + (r + (int64_t)u * RB) * w);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (r + (int64_t)u * RB < r1) acc[0] = O::fold(acc[0], v[u], r + (int64_t)u * RB);
+            }
         }
     }
     // combine the RB row offsets of each column, in row-offset order
